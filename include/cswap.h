@@ -1,0 +1,183 @@
+/*
+ * cswap.h — C ABI of the B200-native CSWAP hot path (libcswap.so).
+ *
+ * CSWAP (Chen et al., CLUSTER'21, /root/reference/PAPER.md) swaps sparse activation tensors
+ * between GPU and host memory and compresses them on the GPU when that is cost-effective:
+ *   - four lossless codecs: ZVC, RLE, CSR, LZ4 (§IV-E);
+ *   - swap-out = compress + D2H to pinned host memory, swap-in = H2D + decompress
+ *     (PAPER.md:120, :228, §IV-A/§V; Fig. 2, :64-:72);
+ *   - a cost model that decides per tensor whether and how to compress
+ *     (§IV-B, Eq. 1-4; codec choice :30; time model §IV-C :164-168).
+ * The byte format of every container is "canonical container v1".
+ *
+ * Conventions (all functions):
+ *   - Plain C types only.  `stream` is a cudaStream_t passed as void* (NULL = legacy default).
+ *   - Device pointers must be CUDA device memory (or host-mapped pinned memory where noted) of
+ *     the device given to cswap_init; tensor and container buffers must be 16-byte aligned.
+ *   - Every call returns a cswap_status and never aborts.  Host-detectable misuse returns
+ *     synchronously; asynchronous kernel-side problems (corrupt containers) are reported through
+ *     a device-visible error word (cswap_decompress) or by cswap_handle_wait (swaps).
+ *   - cswap_last_error() gives a thread-local human-readable detail for the last failure.
+ *   - Elements are raw 32-bit (f32) or 16-bit (f16, bf16) words; "zero" means all bits zero
+ *     (R1), so NaN payloads, -0.0 and denormals round-trip bit-exactly.
+ */
+#ifndef CSWAP_H
+#define CSWAP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  CSWAP_OK = 0,
+  CSWAP_ERR_INVALID = 1,     /* bad argument (null pointer, misalignment, bad dtype/codec/format) */
+  CSWAP_ERR_CUDA = 2,        /* a CUDA runtime call failed; see cswap_last_error() */
+  CSWAP_ERR_NOMEM = 3,       /* device or pinned host allocation failed */
+  CSWAP_ERR_CAPACITY = 4,    /* output buffer smaller than cswap_max_compressed_size() */
+  CSWAP_ERR_CORRUPT = 5,     /* container failed validation */
+  CSWAP_ERR_UNSUPPORTED = 6, /* valid request this build does not implement */
+  CSWAP_ERR_NOT_READY = 7    /* library not initialised */
+} cswap_status;
+
+typedef enum {
+  CSWAP_CODEC_NONE = 0, /* raw copy (vDNN-style uncompressed swap) */
+  CSWAP_CODEC_ZVC = 1,  /* zero-value compression: 1-bit-per-element bitmap + non-zeros */
+  CSWAP_CODEC_RLE = 2,  /* run-length encoding: (length, value) per maximal run */
+  CSWAP_CODEC_CSR = 3,  /* compressed sparse rows of C elements */
+  CSWAP_CODEC_LZ4 = 4,  /* LZ4 block format, canonical greedy parse */
+  CSWAP_CODEC_AUTO = 255 /* cswap_swap_out only: probe + cost model pick one */
+} cswap_codec;
+
+typedef enum { CSWAP_F32 = 0, CSWAP_F16 = 1, CSWAP_BF16 = 2 } cswap_dtype;
+
+/* Format parameters written into every container header.
+ * frame_elems F: > 0, multiple of 1024 (default 4194304).  csr_row C: divides F (default 1024).
+ * lz4_block B: multiple of 1024, <= 65536 (default 65536). */
+typedef struct {
+  uint64_t frame_elems;
+  uint32_t csr_row;
+  uint32_t lz4_block;
+} cswap_format;
+
+/* Sparsity-probe counts: over up to 1024 windows of 256
+ * elements (the whole tensor when n <= 2^18). */
+typedef struct {
+  uint64_t zeros, zero_runs, boundaries, samples, pairs;
+} cswap_probe_result;
+
+/* Cost-model calibration (Table II; time model §IV-C).
+ * Link: t = alpha + bytes / bw per direction (seconds, bytes/s).
+ * beta[codec-1][dir][band][i]: t = b0 + b1*S + b2*S*s, dir 0 = compress, 1 = decompress,
+ * bands [0,.2) [.2,.35) [.35,.5) [.5,.65) [.65,.8) [.8,1] of the probed sparsity s, S = raw bytes.
+ * LZ4 size model: w*nnz + gamma1*zero_runs + gamma2*w*zeros/255.
+ * mode 0 = pipelined (frames overlap codec and copy; margin m), 1 = paper (Eq. 2, m = 0). */
+typedef struct {
+  double alpha_d2h, bw_d2h, alpha_h2d, bw_h2d;
+  double beta[4][2][6][3];
+  double lz4_gamma1, lz4_gamma2;
+  double margin;
+  int32_t mode;
+  int32_t reserved;
+  uint64_t frame_elems; /* F used to predict sizes and pipeline depth */
+  uint32_t csr_row, lz4_block;
+} cswap_calib;
+
+/* Output of the selector: codec (CSWAP_CODEC_NONE or 1..4), predicted T(c*) and T' (s),
+ * per-codec predicted swap time, container bytes, compress and decompress time. */
+typedef struct {
+  int32_t codec;
+  int32_t reserved;
+  double t_pred, t_prime;
+  double t_codec[4];
+  double size[4];
+  double t_c[4], t_dc[4];
+} cswap_decision;
+
+typedef struct cswap_handle cswap_handle; /* opaque, library-owned swap record */
+
+/* ---- lifecycle ---------------------------------------------------------------------------- */
+/* Bind the library to `device` (one device per process), create its internal streams, scratch
+ * and pools, and install built-in calibration defaults.  Idempotent for the same device. */
+cswap_status cswap_init(int device);
+/* Release every resource.  Outstanding handles become invalid. */
+cswap_status cswap_shutdown(void);
+cswap_status cswap_set_calibration(const cswap_calib* calib);
+cswap_status cswap_get_calibration(cswap_calib* out);
+/* Default format used by cswap_swap_out and by calls passing fmt = NULL. */
+cswap_status cswap_set_format(const cswap_format* fmt);
+cswap_status cswap_get_format(cswap_format* out);
+
+/* ---- device codecs (a3-a10) ------------------------------------------------------------------ */
+/* Worst-case container bytes for n elements (0 on invalid arguments).  fmt may be NULL. */
+uint64_t cswap_max_compressed_size(uint64_t n, cswap_dtype dtype, cswap_codec codec, const cswap_format* fmt);
+
+/* Compress n elements at d_in (device) into a container at `out` (device or host-mapped pinned
+ * memory, out_cap bytes >= cswap_max_compressed_size).  Stream-ordered on `stream`; the container
+ * byte count is stored to *out_size (device-visible memory, valid once `stream` reaches it).
+ * codec must be NONE/ZVC/RLE/CSR/LZ4.  d_in is only read. */
+cswap_status cswap_compress(const void* d_in, uint64_t n, cswap_dtype dtype, cswap_codec codec,
+                            const cswap_format* fmt, void* out, uint64_t out_cap, uint64_t* out_size,
+                            void* stream);
+
+/* Decompress the container at `in` (device memory, in_size bytes) into n elements at d_out.
+ * The header is validated on the device: codec, dtype, n and fmt must agree with it.
+ * `err` (device-visible u32, must be 0 on entry; NULL = library word read by
+ * cswap_check_device_error) receives CSWAP_ERR_CORRUPT if validation fails on the device; in
+ * that case d_out's content is unspecified but no out-of-bounds access happens. */
+cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uint64_t n, cswap_dtype dtype,
+                              cswap_codec codec, const cswap_format* fmt, uint32_t* err, void* stream);
+
+/* Synchronise `stream` and return CSWAP_ERR_CORRUPT if a decompress that used err = NULL
+ * reported a problem (the word is then cleared). */
+cswap_status cswap_check_device_error(void* stream);
+
+/* ---- probe + selector (a1, a2) ----------------------------------------------------------------- */
+/* Probe d_in on `stream` and wait for the counts (host result). */
+cswap_status cswap_probe(const void* d_in, uint64_t n, cswap_dtype dtype, cswap_probe_result* out, void* stream);
+/* Pure host function: Eq. 1-4 with the installed (calib = NULL) or given calibration. */
+cswap_status cswap_select_from_probe(uint64_t n, cswap_dtype dtype, const cswap_probe_result* probe,
+                                     double hidden_f, double hidden_b, const cswap_calib* calib,
+                                     cswap_decision* out);
+/* cswap_probe + cswap_select_from_probe with the installed calibration. */
+cswap_status cswap_select(const void* d_in, uint64_t n, cswap_dtype dtype, double hidden_f, double hidden_b,
+                          void* stream, cswap_decision* out);
+
+/* ---- swap pipeline (a11, a12) --------------------------------------------------------------- */
+/* Swap d_in out to library-owned pinned host memory, compressed with `codec` (AUTO: probe +
+ * selector with the given hidden times, PAPER.md:139 Hidden_f/Hidden_b).  Work is ordered after
+ * everything already queued on `stream`.  d_in must stay unmodified until cswap_handle_wait()
+ * returns or cswap_handle_record_out() 's event is waited on. */
+cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, cswap_codec codec, double hidden_f,
+                            double hidden_b, void* stream, cswap_handle** out);
+/* Restore the tensor into d_out (n elements, device), ordered on `stream`: kernels queued on
+ * `stream` afterwards see the restored data.  The handle keeps its host copy (swap-in may be
+ * repeated) until cswap_handle_free. */
+cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream);
+/* Block until every swap operation on h finished; returns deferred asynchronous errors. */
+cswap_status cswap_handle_wait(cswap_handle* h);
+/* Make `stream` wait (device-side) until h's swap-out finished (d_in reusable). */
+cswap_status cswap_handle_record_out(cswap_handle* h, void* stream);
+cswap_status cswap_handle_query(const cswap_handle* h, cswap_codec* codec, uint64_t* container_bytes,
+                                const void** host_container, cswap_decision* decision);
+void cswap_handle_free(cswap_handle* h);
+
+/* ---- calibration (a13) ----------------------------------------------------------------------- */
+/* Ordinary least squares t = b0 + b1*S + b2*S*s over m samples ("linear
+ * regression"); beta_out[3].  Returns CSWAP_ERR_INVALID if m < 3 or the design is singular. */
+cswap_status cswap_fit_time_model(const double* S, const double* s, const double* t, uint64_t m, double* beta_out);
+/* Ordinary least squares t = alpha + bytes / bw (link model); alpha_out, bw_out. */
+cswap_status cswap_fit_link(const double* bytes, const double* t, uint64_t m, double* alpha_out, double* bw_out);
+
+/* ---- diagnostics ---------------------------------------------------------------------------- */
+const char* cswap_status_string(cswap_status s);
+const char* cswap_last_error(void);
+/* Number of kernels this library launched since init (for bench accounting). */
+uint64_t cswap_kernel_launches(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CSWAP_H */

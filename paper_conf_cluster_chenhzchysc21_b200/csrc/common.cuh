@@ -1,0 +1,172 @@
+// common.cuh — shared device helpers for the CSWAP sm_100a kernels.
+//
+// Container v1 geometry, the epoch-tagged decoupled-lookback protocol used by
+// the single-pass codec kernels, and small PTX wrappers (acquire/release at .gpu scope).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace cswap {
+
+constexpr int kThreads = 256;          // every tile kernel: 8 warps
+constexpr int kWarps = kThreads / 32;
+constexpr uint32_t kTileBytes = 32768; // one tile = 32 KiB of raw input (8192 f32 / 16384 f16)
+constexpr uint32_t kEpochs = 1u << 14; // status epoch tag width (14 bits)
+
+enum : int { kNone = 0, kZVC = 1, kRLE = 2, kCSR = 3, kLZ4 = 4 };
+enum : uint32_t { kErrOK = 0, kErrCorrupt = 5 };
+
+__host__ __device__ __forceinline__ uint64_t a16(uint64_t x) { return (x + 15) & ~uint64_t(15); }
+__host__ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__host__ __device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a > b ? a : b; }
+__host__ __device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+__host__ __device__ __forceinline__ uint64_t data_start(uint32_t K) { return a16(64 + 8ull * K); }
+__host__ __device__ __forceinline__ uint64_t frame_len(uint64_t n, uint64_t F, uint64_t k) {
+  uint64_t s = k * F;
+  return (n - s) < F ? (n - s) : F;
+}
+
+// ---- scratch shared by one launch sequence (owned by the runtime, see runtime.cpp) ----
+struct Scratch {
+  uint64_t* status;       // per-tile lookback word: value<<16 | epoch<<2 | flag
+  uint32_t* tickets;      // per-epoch tile-ticket counters (zeroed slots)
+  uint64_t* aux;          // per-frame / per-block u64 scratch (frame starts, block offsets ...)
+  uint64_t* aux2;         // second per-frame / per-tile array
+  uint32_t* err;          // device error word (first error wins)
+  uint64_t cap_tiles, cap_aux;
+};
+
+// ---- memory-order helpers -------------------------------------------------------------
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(uint64_t* p, uint64_t v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_acquire32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+constexpr uint64_t kFlagA = 1, kFlagP = 2;
+__device__ __forceinline__ uint64_t make_status(uint64_t value, uint32_t epoch, uint64_t flag) {
+  return (value << 16) | (uint64_t(epoch) << 2) | flag;
+}
+__device__ __forceinline__ uint32_t status_flag(uint64_t s, uint32_t epoch) {
+  return (uint32_t(s >> 2) & (kEpochs - 1)) == epoch ? uint32_t(s & 3) : 0u;
+}
+__device__ __forceinline__ uint64_t status_value(uint64_t s) { return s >> 16; }
+
+__device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// Decoupled lookback (single-pass chained scan, CUB style) for tile `tile` inside a segment
+// whose first tile is `seg_first` (< tile).  The segment's first tile publishes only P.
+// Called by one full warp; returns the exclusive prefix (sum of A values + the nearest P).
+__device__ __forceinline__ uint64_t lookback(const uint64_t* status, int64_t tile, int64_t seg_first,
+                                             uint32_t epoch) {
+  const int lane = threadIdx.x & 31;
+  uint64_t excl = 0;
+  int64_t pos = tile - 1;
+  while (true) {
+    const int64_t t = pos - lane;
+    uint64_t s = 0;
+    uint32_t f = 0;
+    bool ok;
+    do {
+      if (t >= seg_first) {
+        s = ld_acquire(status + t);
+        f = status_flag(s, epoch);
+        ok = f != 0;
+      } else {
+        ok = true;  // below the segment: contributes nothing (a P is always found first)
+        f = 0;
+        s = 0;
+      }
+    } while (!__all_sync(0xffffffffu, ok));
+    const uint32_t pmask = __ballot_sync(0xffffffffu, t >= seg_first && f == kFlagP);
+    if (pmask) {
+      const int pl = __ffs(pmask) - 1;  // nearest P
+      uint64_t v = (lane <= pl && t >= seg_first) ? status_value(s) : 0;
+      excl += warp_sum_u64(v);
+      return excl;
+    }
+    uint64_t v = (t >= seg_first) ? status_value(s) : 0;
+    excl += warp_sum_u64(v);
+    pos -= 32;
+  }
+}
+
+__device__ __forceinline__ void set_error(uint32_t* err, uint32_t code) {
+  if (err) atomicCAS(err, 0u, code);
+}
+
+// ---- bulk async copy (TMA 1-D: cp.async.bulk global -> shared, mbarrier completion) -----
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(bar));
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(bar));
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(a), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+  uint32_t d = static_cast<uint32_t>(__cvta_generic_to_shared(smem_dst));
+  uint32_t b = static_cast<uint32_t>(__cvta_generic_to_shared(bar));
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(d),
+      "l"(gsrc), "r"(bytes), "r"(b)
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+  uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(bar));
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(a),
+      "r"(phase)
+      : "memory");
+}
+
+// ---- vector helpers -------------------------------------------------------------------
+__device__ __forceinline__ uint4 ldg_stream(const uint4* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void stg_stream(uint4* p, uint4 v) {
+  asm volatile("st.global.L1::no_allocate.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w)
+               : "memory");
+}
+
+// Write the 64-byte container header (one thread).
+__device__ __forceinline__ void write_header(uint8_t* out, int codec, int dtype, uint64_t n, uint64_t F,
+                                             uint32_t K, uint32_t param, uint64_t total) {
+  uint32_t* o32 = reinterpret_cast<uint32_t*>(out);
+  uint64_t* o64 = reinterpret_cast<uint64_t*>(out);
+  o32[0] = 0x50575343u;                                             // "CSWP"
+  o32[1] = 1u | (uint32_t(codec) << 16) | (uint32_t(dtype) << 24);  // version 1, codec, dtype
+  o64[1] = n;
+  o64[2] = F;
+  o32[6] = K;
+  o32[7] = param;
+  o64[4] = total;
+  o64[5] = 0;
+  o64[6] = 0;
+  o64[7] = 0;
+}
+
+}  // namespace cswap

@@ -1,0 +1,208 @@
+// container.cu — codec-independent kernels: container header/prep, NONE frames, sparsity probe.
+//
+// Container v1 layout: DESIGN.md §3.  Probe: PAPER.md:118 (§IV-A, the tensor profiler collects
+// sparsity), :327 (§V-E, "CSWAP utilizes GPU multi-cores to profile tensor sparsity"); window
+// design DESIGN.md R15 / §3.3.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace cswap {
+
+// ---- header-only container (n = 0) and NONE header ------------------------------------------
+__global__ void header_kernel(uint8_t* out, int codec, int dtype, uint64_t n, uint64_t F, uint32_t param,
+                              uint64_t* out_size) {
+  const uint32_t K = uint32_t(cdiv(n, F));
+  const int w = dtype == 0 ? 4 : 2;
+  uint64_t total = data_start(K);
+  for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) {
+    const uint64_t fb = a16(uint64_t(w) * frame_len(n, F, k));
+    reinterpret_cast<uint64_t*>(out + 64)[k] = fb;
+  }
+  if (threadIdx.x == 0) {
+    for (uint32_t k = 0; k < K; k++) total += a16(uint64_t(w) * frame_len(n, F, k));
+    write_header(out, codec, dtype, n, F, K, param, total);
+    for (uint64_t b = 64 + 8ull * K; b < data_start(K); b += 8) *reinterpret_cast<uint64_t*>(out + b) = 0;
+    if (K) {  // zero the pad after the last raw frame
+      const uint64_t end = data_start(K) + uint64_t(w) * n;
+      for (uint64_t b = end; b < total; b++) out[b] = 0;
+    }
+    *out_size = total;
+  }
+}
+
+cudaError_t launch_header_only(uint8_t* out, int codec, int dtype, uint64_t F, uint32_t param, uint64_t* out_size,
+                               cudaStream_t st) {
+  header_kernel<<<1, 32, 0, st>>>(out, codec, dtype, 0, F, param, out_size);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, int dtype, uint8_t* out,
+                                 uint64_t* out_size, cudaStream_t st) {
+  const uint32_t K = uint32_t(cdiv(n, F));
+  // non-last frames are F*w bytes (a multiple of 16), so the raw frames are one contiguous run
+  cudaError_t e = cudaMemcpyAsync(out + data_start(K), in, n * w, cudaMemcpyDeviceToDevice, st);
+  if (e != cudaSuccess) return e;
+  header_kernel<<<1, 256, 0, st>>>(out, kNone, dtype, n, F, 0, out_size);
+  return cudaGetLastError();
+}
+
+// ---- prep: validate the header and scan the frame table --------------------------------------
+__device__ __forceinline__ uint64_t block_excl_scan_u64(uint64_t v, uint64_t* s_warp, uint64_t* total) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  uint64_t inc = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+    if (lane >= o) inc += y;
+  }
+  if (lane == 31) s_warp[warp] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint64_t acc = 0;
+    for (int w = 0; w < nw; w++) {
+      uint64_t x = s_warp[w];
+      s_warp[w] = acc;
+      acc += x;
+    }
+    s_warp[nw] = acc;
+  }
+  __syncthreads();
+  const uint64_t r = s_warp[warp] + inc - v;
+  *total = s_warp[nw];
+  __syncthreads();
+  return r;
+}
+
+__global__ void __launch_bounds__(1024) prep_kernel(const uint8_t* in, uint64_t in_size, int codec, int dtype,
+                                                    uint64_t n, uint64_t F, uint32_t param, uint64_t* fstart,
+                                                    uint64_t* fbytes, uint32_t* err) {
+  __shared__ int s_ok;
+  __shared__ uint64_t s_total;
+  __shared__ uint64_t s_warp[33];
+  const uint32_t K = uint32_t(cdiv(n, F));
+  if (threadIdx.x == 0) {
+    int ok = in_size >= 64;
+    if (ok) {
+      const uint32_t* h32 = reinterpret_cast<const uint32_t*>(in);
+      const uint64_t* h64 = reinterpret_cast<const uint64_t*>(in);
+      ok = h32[0] == 0x50575343u && (h32[1] & 0xFFFFu) == 1u && int((h32[1] >> 16) & 0xFF) == codec &&
+           int(h32[1] >> 24) == dtype && h64[1] == n && h64[2] == F && h32[6] == K && h32[7] == param;
+      s_total = h64[4];
+      ok = ok && s_total <= in_size && s_total >= data_start(K);
+    }
+    s_ok = ok;
+    if (!ok) set_error(err, kErrCorrupt);
+  }
+  __syncthreads();
+  if (!s_ok) return;
+  const uint64_t* table = reinterpret_cast<const uint64_t*>(in + 64);
+  const uint64_t base = data_start(K);
+  uint64_t carry = 0;
+  bool bad = false;
+  for (uint32_t c = 0; c < K; c += blockDim.x) {
+    const uint32_t k = c + threadIdx.x;
+    const uint64_t fb = k < K ? table[k] : 0;
+    bad |= (fb & 15) != 0 || fb > s_total;
+    uint64_t tot;
+    const uint64_t ex = block_excl_scan_u64(fb, s_warp, &tot);
+    if (k < K) {
+      fstart[k] = base + carry + ex;
+      fbytes[k] = fb;
+    }
+    carry += tot;
+  }
+  if (bad) set_error(err, kErrCorrupt);
+  if (threadIdx.x == 0 && base + carry != s_total) set_error(err, kErrCorrupt);
+}
+
+cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
+                        uint32_t param, const Scratch& sc, uint32_t* err, cudaStream_t st) {
+  prep_kernel<<<1, 1024, 0, st>>>(in, in_size, codec, dtype, n, F, param, sc.aux, sc.aux2, err);
+  return cudaGetLastError();
+}
+
+// ---- NONE decompress: frames are raw; check sizes, copy -----------------------------------
+__global__ void none_check_kernel(uint64_t n, uint64_t F, int w, const uint64_t* fbytes, uint32_t* err) {
+  const uint32_t K = uint32_t(cdiv(n, F));
+  for (uint32_t k = threadIdx.x; k < K; k += blockDim.x)
+    if (fbytes[k] != a16(uint64_t(w) * frame_len(n, F, k))) set_error(err, kErrCorrupt);
+}
+
+cudaError_t launch_none_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, const Scratch& sc,
+                                   uint32_t* err, cudaStream_t st) {
+  const uint32_t K = uint32_t(cdiv(n, F));
+  none_check_kernel<<<1, 256, 0, st>>>(n, F, w, sc.aux2, err);
+  return cudaMemcpyAsync(out, in + data_start(K), n * w, cudaMemcpyDeviceToDevice, st);
+}
+
+// ---- sparsity probe ----------------------------------------------------------------------
+constexpr int kProbeW = 256, kProbeSw = 1024;
+
+template <typename T>
+__global__ void __launch_bounds__(kThreads) probe_kernel(const T* __restrict__ x, uint64_t n, uint32_t pieces,
+                                                         bool single, uint64_t* partial, uint32_t* done,
+                                                         uint64_t* counts3) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t z = 0, zr = 0, bd = 0;
+  for (uint32_t p = blockIdx.x * kWarps + warp; p < pieces; p += gridDim.x * kWarps) {
+    uint64_t start, ws;
+    if (single) { start = uint64_t(p) * kProbeW; ws = 0; }
+    else { start = uint64_t(p) * (n - kProbeW) / (kProbeSw - 1); ws = start; }
+    const uint64_t end = single ? umin64(start + kProbeW, n) : start + kProbeW;
+    uint32_t v[8];
+    const uint64_t i0 = start + lane * 8;
+#pragma unroll
+    for (int i = 0; i < 8; i++) v[i] = (i0 + i < end) ? uint32_t(x[i0 + i]) : 0u;
+    uint32_t prev = __shfl_up_sync(0xffffffffu, v[7], 1);
+    if (lane == 0) prev = start > ws ? uint32_t(x[start - 1]) : 0u;
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+      const uint64_t gi = i0 + i;
+      if (gi < end) {
+        const bool first = gi == ws;
+        z += v[i] == 0;
+        zr += v[i] == 0 && (first || prev != 0);
+        bd += !first && v[i] != prev;
+      }
+      prev = v[i];
+    }
+  }
+  z = warp_sum_u64(z);
+  zr = warp_sum_u64(zr);
+  bd = warp_sum_u64(bd);
+  __shared__ uint64_t s[kWarps][3];
+  __shared__ bool s_last;
+  if (lane == 0) { s[warp][0] = z; s[warp][1] = zr; s[warp][2] = bd; }
+  __syncthreads();
+  if (threadIdx.x < 3) {
+    uint64_t a = 0;
+    for (int w = 0; w < kWarps; w++) a += s[w][threadIdx.x];
+    partial[blockIdx.x * 3 + threadIdx.x] = a;
+  }
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) s_last = atomicAdd(done, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (s_last && threadIdx.x < 3) {
+    __threadfence();
+    uint64_t a = 0;
+    for (uint32_t b = 0; b < gridDim.x; b++) a += reinterpret_cast<volatile uint64_t*>(partial)[b * 3 + threadIdx.x];
+    counts3[threadIdx.x] = a;
+  }
+}
+
+cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, const Scratch& sc, uint32_t epoch,
+                         cudaStream_t st) {
+  const bool single = n <= uint64_t(kProbeW) * kProbeSw;
+  const uint32_t pieces = single ? uint32_t(cdiv(n, kProbeW)) : kProbeSw;
+  const uint32_t grid = uint32_t(umin64(cdiv(pieces, kWarps), 128));
+  if (w == 4)
+    probe_kernel<uint32_t><<<grid, kThreads, 0, st>>>(static_cast<const uint32_t*>(in), n, pieces, single, sc.aux2,
+                                                      sc.tickets + epoch, counts3);
+  else
+    probe_kernel<uint16_t><<<grid, kThreads, 0, st>>>(static_cast<const uint16_t*>(in), n, pieces, single, sc.aux2,
+                                                      sc.tickets + epoch, counts3);
+  return cudaGetLastError();
+}
+
+}  // namespace cswap

@@ -1,0 +1,49 @@
+// kernels.h — internal launchers (not part of the public C ABI; see include/cswap.h).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+
+namespace cswap {
+
+// container.cu
+cudaError_t launch_header_only(uint8_t* out, int codec, int dtype, uint64_t F, uint32_t param, uint64_t* out_size,
+                               cudaStream_t st);
+cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
+                        uint32_t param, const Scratch& sc, uint32_t* err, cudaStream_t st);
+cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, int dtype, uint8_t* out,
+                                 uint64_t* out_size, cudaStream_t st);
+cudaError_t launch_none_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, const Scratch& sc,
+                                   uint32_t* err, cudaStream_t st);
+cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, const Scratch& sc, uint32_t epoch,
+                         cudaStream_t st);
+
+// zvc.cu
+uint32_t zvc_tiles(uint64_t n, int w, uint64_t F, uint32_t k0, uint32_t k1, uint32_t* tpf_out);
+cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
+                                const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st);
+cudaError_t launch_zvc_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
+                                  uint32_t k1, const Scratch& sc, uint32_t epoch, uint32_t* err, cudaStream_t st);
+
+// rle.cu
+uint32_t rle_tiles(uint64_t n, int w, uint64_t F);
+cudaError_t launch_rle_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
+                                const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st);
+cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
+                                  uint32_t k1, const Scratch& sc, uint32_t epoch, uint32_t* err, cudaStream_t st);
+
+// csr.cu
+cudaError_t launch_csr_compress(const void* in, uint64_t n, int w, uint64_t F, uint32_t C, uint8_t* out,
+                                uint64_t* out_size, const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st);
+cudaError_t launch_csr_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t C,
+                                  uint32_t k0, uint32_t k1, const Scratch& sc, uint32_t* err, cudaStream_t st);
+
+// lz4.cu
+uint64_t lz4_scratch_bytes(uint64_t n, int w, uint64_t F, uint32_t B);
+cudaError_t launch_lz4_compress(const void* in, uint64_t n, int w, uint64_t F, uint32_t B, uint8_t* out,
+                                uint64_t* out_size, uint8_t* slots, const Scratch& sc, int dtype, cudaStream_t st);
+cudaError_t launch_lz4_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t B,
+                                  uint32_t k0, uint32_t k1, const Scratch& sc, uint32_t* err, cudaStream_t st);
+
+}  // namespace cswap

@@ -1,0 +1,204 @@
+// select.cpp — execution advisor: the swap cost model of PAPER.md §IV-B (Eq. 1-4, :137-154),
+// the codec choice of :30, and the LR time model of §IV-C (:164-168).  Host code, double
+// precision, evaluation order fixed by DESIGN.md §3.3 (so the CPU oracle can be compared exactly).
+#include <cmath>
+#include <cstdint>
+#include <cstring>
+#include <vector>
+
+#include "../../include/cswap.h"
+#include "internal.h"
+
+namespace cswap {
+
+namespace {
+inline uint64_t al16(uint64_t x) { return (x + 15) / 16 * 16; }
+inline uint64_t cd(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+inline int band(double s) {
+  static const double edges[5] = {0.2, 0.35, 0.5, 0.65, 0.8};  // DESIGN.md R14
+  int b = 0;
+  while (b < 5 && s >= edges[b]) b++;
+  return b;
+}
+}  // namespace
+
+ProbeEstimates estimate(uint64_t n, const cswap_probe_result& p) {
+  ProbeEstimates e{};
+  if (p.samples == 0) {
+    e.runs = n ? 1 : 0;
+    return e;
+  }
+  const uint64_t half = p.samples / 2;
+  e.zeros = (p.zeros * n + half) / p.samples;  // u64 round-half-up (R19)
+  e.nnz = n - e.zeros;
+  e.runs = p.pairs ? 1 + (p.boundaries * (n - 1) + p.pairs / 2) / p.pairs : 1;
+  e.zero_runs = (p.zero_runs * n + half) / p.samples;
+  return e;
+}
+
+void decide(uint64_t n, int w, const cswap_probe_result& p, double hf, double hb, const cswap_calib& c,
+            cswap_decision* out) {
+  std::memset(out, 0, sizeof(*out));
+  out->codec = CSWAP_CODEC_NONE;
+  if (n == 0 || p.samples == 0) return;
+  const ProbeEstimates e = estimate(n, p);
+  const bool paper = c.mode == 1;
+  const double S = double(n) * double(w);
+  const double s = double(p.zeros) / double(p.samples);
+  const int b = band(s);
+  const double ad = paper ? 0.0 : c.alpha_d2h, ah = paper ? 0.0 : c.alpha_h2d;
+  const uint64_t F = c.frame_elems, K = cd(n, F);
+  const uint64_t hdr = al16(64 + 8 * K);
+
+  auto xd = [&](double bytes) { return ad + bytes / c.bw_d2h; };
+  auto xh = [&](double bytes) { return ah + bytes / c.bw_h2d; };
+  // Eq. 1: swap cost without compression
+  const double Tp = std::fmax(xd(S) - hf, 0.0) + std::fmax(xh(S) - hb, 0.0);
+
+  // per-frame fixed section bytes of each codec (exact container geometry)
+  uint64_t fix[4] = {0, 0, 0, 0};
+  for (uint64_t k = 0; k < K; k++) {
+    const uint64_t Fk = (k + 1) * F <= n ? F : n - k * F;
+    fix[0] += al16(4 * cd(Fk, 32));
+    fix[1] += 16;
+    fix[2] += al16(4 * (cd(Fk, c.csr_row) + 1));
+    fix[3] += al16(4 * cd(Fk * uint64_t(w), c.lz4_block));
+  }
+  double best = 0.0;
+  int best_c = 0;
+  for (int ci = 0; ci < 4; ci++) {
+    const double* bc = c.beta[ci][0][b];
+    const double* bd = c.beta[ci][1][b];
+    const double tc = bc[0] + bc[1] * S + bc[2] * S * s;
+    const double tdc = bd[0] + bd[1] * S + bd[2] * S * s;
+    double size;
+    if (paper) {
+      size = S * (1.0 - s);  // Eq. 3-4: Size x (1 - Sparsity)
+    } else if (ci == 0) {    // ZVC
+      size = double(hdr + fix[0] + al16(e.nnz * w));
+    } else if (ci == 1) {    // RLE
+      uint64_t r = e.runs + (K - 1);
+      if (r > n) r = n;
+      size = double(hdr + fix[1] + al16(4 * r) + al16(r * w));
+    } else if (ci == 2) {    // CSR
+      size = double(hdr + fix[2] + al16(4 * e.nnz) + al16(e.nnz * w));
+    } else {                 // LZ4
+      size = double(hdr + fix[3]) + double(e.nnz * w) + c.lz4_gamma1 * double(e.zero_runs) +
+             c.lz4_gamma2 * double(w) * double(e.zeros) / 255.0;
+    }
+    const double xo = xd(size), xi = xh(size);
+    double T;
+    if (paper) {
+      T = tc + tdc + std::fmax(xo - hf, 0.0) + std::fmax(xi - hb, 0.0);  // Eq. 2
+    } else {
+      const double Kd = double(K);
+      const double Tout = std::fmax(tc, xo) + std::fmin(tc, xo) / Kd;
+      const double Tin = std::fmax(tdc, xi) + std::fmin(tdc, xi) / Kd;
+      T = std::fmax(Tout - hf, 0.0) + std::fmax(Tin - hb, 0.0);
+    }
+    out->t_codec[ci] = T;
+    out->size[ci] = size;
+    out->t_c[ci] = tc;
+    out->t_dc[ci] = tdc;
+    if (ci == 0 || T < best) {
+      best = T;
+      best_c = ci + 1;
+    }
+  }
+  const double m = paper ? 0.0 : c.margin;
+  out->t_pred = best;
+  out->t_prime = Tp;
+  out->codec = best < (1.0 - m) * Tp ? best_c : CSWAP_CODEC_NONE;  // PAPER.md:137, strict
+}
+
+// OLS by modified Gram-Schmidt on column-scaled [1, S, S*s] (robust for S ~ 1e9).
+bool fit3(const double* S, const double* s, const double* t, uint64_t m, double* beta) {
+  if (m < 3) return false;
+  double scale[3] = {1.0, 0.0, 0.0};
+  for (uint64_t i = 0; i < m; i++) {
+    scale[1] = std::fmax(scale[1], std::fabs(S[i]));
+    scale[2] = std::fmax(scale[2], std::fabs(S[i] * s[i]));
+  }
+  if (scale[1] == 0) scale[1] = 1;
+  if (scale[2] == 0) scale[2] = 1;
+  std::vector<double> Q(3 * m);
+  for (uint64_t i = 0; i < m; i++) {
+    Q[i] = 1.0;
+    Q[m + i] = S[i] / scale[1];
+    Q[2 * m + i] = S[i] * s[i] / scale[2];
+  }
+  double R[3][3] = {{0}};
+  for (int jc = 0; jc < 3; jc++) {
+    double* qj = &Q[jc * m];
+    for (int ic = 0; ic < jc; ic++) {
+      const double* qi = &Q[ic * m];
+      double dot = 0;
+      for (uint64_t r = 0; r < m; r++) dot += qi[r] * qj[r];
+      R[ic][jc] = dot;
+      for (uint64_t r = 0; r < m; r++) qj[r] -= dot * qi[r];
+    }
+    double nrm = 0;
+    for (uint64_t r = 0; r < m; r++) nrm += qj[r] * qj[r];
+    nrm = std::sqrt(nrm);
+    R[jc][jc] = nrm;
+    if (nrm < 1e-12 * std::sqrt(double(m))) return false;
+    for (uint64_t r = 0; r < m; r++) qj[r] /= nrm;
+  }
+  double qt[3];
+  for (int jc = 0; jc < 3; jc++) {
+    double dot = 0;
+    for (uint64_t r = 0; r < m; r++) dot += Q[jc * m + r] * t[r];
+    qt[jc] = dot;
+  }
+  double x[3];
+  for (int jc = 2; jc >= 0; jc--) {
+    double v = qt[jc];
+    for (int kc = jc + 1; kc < 3; kc++) v -= R[jc][kc] * x[kc];
+    x[jc] = v / R[jc][jc];
+  }
+  for (int jc = 0; jc < 3; jc++) beta[jc] = x[jc] / scale[jc];
+  return true;
+}
+
+bool fit_link(const double* bytes, const double* t, uint64_t m, double* alpha, double* bw) {
+  if (m < 2) return false;
+  double mb = 0, mt = 0;
+  for (uint64_t i = 0; i < m; i++) { mb += bytes[i]; mt += t[i]; }
+  mb /= double(m);
+  mt /= double(m);
+  double sbb = 0, sbt = 0;
+  for (uint64_t i = 0; i < m; i++) {
+    sbb += (bytes[i] - mb) * (bytes[i] - mb);
+    sbt += (bytes[i] - mb) * (t[i] - mt);
+  }
+  if (sbb <= 0 || sbt <= 0) return false;
+  const double slope = sbt / sbb;
+  *bw = 1.0 / slope;
+  *alpha = mt - slope * mb;
+  return true;
+}
+
+void default_calib(cswap_calib* c) {
+  std::memset(c, 0, sizeof(*c));
+  // Placeholder until calibration runs on the box (bench.py --calibrate writes calib/b200.json):
+  // PCIe Gen5 x16 pinned copies ~50 GB/s per direction with ~10 us fixed cost; codecs at
+  // ~2 TB/s of raw bytes with ~10 us fixed cost (LZ4 compress ~100 GB/s).
+  c->alpha_d2h = c->alpha_h2d = 10e-6;
+  c->bw_d2h = c->bw_h2d = 50e9;
+  for (int ci = 0; ci < 4; ci++)
+    for (int d = 0; d < 2; d++)
+      for (int b = 0; b < 6; b++) {
+        c->beta[ci][d][b][0] = 10e-6;
+        c->beta[ci][d][b][1] = (ci == 3 && d == 0) ? 1.0 / 100e9 : 1.0 / 2e12;
+        c->beta[ci][d][b][2] = 0.0;
+      }
+  c->lz4_gamma1 = 3.0;
+  c->lz4_gamma2 = 1.0;
+  c->margin = 0.05;
+  c->mode = 0;
+  c->frame_elems = uint64_t(1) << 22;
+  c->csr_row = 1024;
+  c->lz4_block = 65536;
+}
+
+}  // namespace cswap
