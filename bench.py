@@ -1,0 +1,487 @@
+"""bench.py — CSWAP hot path on B200: compressed swap-out + swap-in of the VGG16 batch-64
+activation set (BASELINE.json configs[2]) with cost-model codec selection.
+
+One step = the whole hot path over one batch: for each of the 12 conv-input ReLU/MAX tensors
+in forward order, probe + select + compress + D2H to pinned host (swap-out); then for each in
+reverse order, H2D + decompress (swap-in) (Fig. 2, :64-:72; vDNN policy :251).
+value = raw tensor bytes swapped out and back in per second, summed over ranks (GB/s).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload vgg16|resnet50|bert] [--calibrate] [--no-extras]
+Multi-GPU: one process per GPU under torchrun; each rank swaps its own replica of the set
+(no collective on the data path, "scaling": "weak"); time = max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "compressed swap-out+in latency & codec GB/s vs HBM roofline, 1/2/4/8 B200"
+CALIB_PATH = os.path.join(ROOT, "calib", "b200.json")
+NCU_SUMMARY = os.path.join(ROOT, "profiles", "ncu_zvc_r01.json")
+
+
+def log(*a):
+    if int(os.environ.get("RANK", "0")) == 0:
+        print(*a, file=sys.stderr, flush=True)
+
+
+def workload(name: str):
+    import synth
+    if name == "vgg16":
+        return "vgg16_b64_swapset", synth.vgg16_b64(), synth.F32
+    if name == "resnet50":
+        return "resnet50_b64_swapset", synth.resnet50_b64(), synth.F32
+    if name == "bert":
+        return "bert_large_b8_swapset", synth.bert_large_b8(), synth.F16
+    raise SystemExit(f"unknown workload {name}")
+
+
+# ------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    FIELDS = ["clocks.sm", "clocks.max.sm", "clocks_event_reasons.hw_slowdown",
+              "clocks_event_reasons.hw_thermal_slowdown", "clocks_event_reasons.sw_thermal_slowdown",
+              "clocks_event_reasons.sw_power_cap"]
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), "--query-gpu=" + ",".join(self.FIELDS),
+                 "--format=csv,noheader,nounits", "-lms", "200"], stdout=subprocess.PIPE,
+                stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        self.out = ""
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.out, _ = self.proc.communicate(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self) -> dict:
+        sms, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in (getattr(self, "out", "") or "").splitlines():
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) != len(self.FIELDS):
+                continue
+            try:
+                sms.append(float(parts[0]))
+                mx = float(parts[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[2:]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sms) if sms else None, "sm_max_mhz": mx, "samples": len(sms),
+                "reasons": sorted(reasons)}
+
+
+# ------------------------------------------------------------------------------------ ours
+def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
+    import torch
+
+    import synth
+    from paper_conf_cluster_chenhzchysc21_b200 import calibrate, cswap as C
+
+    torch.cuda.set_device(local_rank)
+    C.init(local_rank)
+    codecs_built = [c for c in (C.ZVC, C.RLE, C.CSR, C.LZ4) if _codec_built(C, c)]
+    if args.calibrate or not calibrate.load(CALIB_PATH):
+        log(f"calibrating on the box (codecs {codecs_built}) ...")
+        calibrate.run(codecs_built, quick=not args.calibrate, path=CALIB_PATH if args.calibrate else None, log=log)
+    cal = C.get_calibration()
+
+    wname, tensors_spec, dtype = workload(args.workload)
+    w = C.WIDTH[dtype]
+    dev = torch.device("cuda", local_rank)
+    tensors, outs, sizes = [], [], []
+    for i, (name, shape, s) in enumerate(tensors_spec):
+        n = synth.numel(shape)
+        tensors.append(synth.relu_iid_torch(n, s, seed=synth.seed_of(3, 0, 0, i) + 7919 * rank, dtype=dtype,
+                                            device=dev))
+        outs.append(torch.empty_like(tensors[-1]))
+        sizes.append(n)
+    raw_bytes = sum(sizes) * w
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+
+    def step(codec):
+        hs = [C.swap_out(t, n, dtype, codec) for t, n in zip(tensors, sizes)]
+        for o, h in zip(reversed(outs), reversed(hs)):
+            h.swap_in(o)
+        return hs
+
+    def barrier():
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def timed(codec, steps, warmup, record=False, clocks=False):
+        for _ in range(warmup):
+            for h in step(codec):
+                h.close()
+        barrier()
+        launches0 = C.kernel_launches()
+        if record:
+            C.collect_kernel_timing()
+            C.set_kernel_timing(True)
+        sampler = ClockSampler(local_rank) if clocks else None
+        if sampler:
+            sampler.__enter__()
+        t0 = time.perf_counter()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        hs_last = None
+        for i in range(steps):
+            hs = step(codec)
+            if i + 1 < steps:
+                for h in hs:
+                    h.close()
+            else:
+                hs_last = hs
+        b.record(stream)
+        b.synchronize()
+        wall = time.perf_counter() - t0
+        if sampler:
+            sampler.__exit__(None, None, None)
+        if record:
+            C.set_kernel_timing(False)
+        launches = C.kernel_launches() - launches0
+        ms = a.elapsed_time(b)
+        recs = C.collect_kernel_timing() if record else []
+        barrier()
+        info = [h.query() for h in hs_last]
+        for h in hs_last:
+            h.close()
+        return {"ms": ms, "wall_s": wall, "launches": launches, "records": recs, "handles": info,
+                "clocks": sampler.summary() if sampler else None}
+
+    # ---- headline: AUTO selection ---------------------------------------------------------
+    main = timed(C.AUTO, args.steps, args.warmup, record=True, clocks=True)
+    ms_max = _max_over_ranks(main["ms"], dist)
+    ms_per_step = ms_max / args.steps
+    value = world * raw_bytes / (ms_per_step * 1e-3) / 1e9
+    for o, t in zip(outs, tensors):  # the last step restored every tensor bitwise
+        assert torch.equal(o, t), "swap round trip mismatch"
+
+    roof = _roofline(main["records"])
+    result = {
+        "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32" if w == 4 else "u16", "data": "synthetic",
+        "config": {"workload": wname, "tensors": len(sizes), "raw_MiB_per_gpu": raw_bytes / 2**20,
+                   "elem": synth.NAMES[dtype], "selector": "pipelined" if cal.mode == 0 else "paper",
+                   "frame_elems": int(C.get_format().frame_elems),
+                   "l2": "working set 2.2 GB >> 126 MB L2: every step streams from HBM (no flush needed)",
+                   "parallelism": f"replicas x{world}"},
+        "gpu_launches": main["launches"],
+        "clocks": main["clocks"],
+        "roofline": roof,
+    }
+    decisions = [q["codec"] for q in main["handles"]]
+    comp_bytes = [q["bytes"] for q in main["handles"]]
+    result["config"]["codecs_chosen"] = [C.CODEC_NAMES[c] for c in decisions]
+    result["config"]["compressed_MiB"] = sum(comp_bytes) / 2**20
+
+    if not args.no_extras:
+        result["extras"] = _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, raw_bytes,
+                                   world)
+        result["e2e"] = _e2e(args, C, torch, tensors, outs, sizes, dtype, w, dist, world, stream)
+    if rank == 0 and world == 1 and not args.no_cpu:
+        result["cpu_baseline"] = _cpu_baseline(tensors, sizes, decisions, dtype)
+    return result
+
+
+def _codec_built(C, codec) -> bool:
+    import torch
+    x = torch.zeros(1024, dtype=torch.int32, device="cuda")
+    cap = C.max_compressed_size(1024, C.F32, codec)
+    buf = torch.empty(cap, dtype=torch.uint8, device="cuda")
+    sz = torch.zeros(1, dtype=torch.int64, device="cuda")
+    try:
+        C.compress(x, 1024, C.F32, codec, buf, cap, sz)
+        torch.cuda.synchronize()
+        return True
+    except C.CswapError as e:
+        if e.status == 6:
+            return False
+        raise
+
+
+def _max_over_ranks(v: float, dist) -> float:
+    if dist is None:
+        return v
+    import torch
+    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d.get("hbm_gbs", 6650.0), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def _roofline(records) -> dict:
+    """Dominant kernel = the codec launch group with the largest total device time in the timed
+    region; algorithmic bytes = raw bytes + container bytes per launch."""
+    peak, src = _peaks()
+    groups = {}
+    for r in records:
+        if r["direction"] == 2:
+            continue
+        key = (r["codec"], r["direction"])
+        g = groups.setdefault(key, {"ms": 0.0, "bytes": 0, "launches": 0})
+        g["ms"] += r["ms"]
+        g["bytes"] += r["raw_bytes"] + r["comp_bytes"]
+        g["launches"] += 1
+    if not groups:
+        return {"bound": "hbm", "achieved": None, "peak": peak, "unit": "GB/s", "frac": None, "traffic": None}
+    (codec, d), g = max(groups.items(), key=lambda kv: kv[1]["ms"])
+    achieved = g["bytes"] / (g["ms"] * 1e-3) / 1e9
+    names = {0: "none", 1: "zvc", 2: "rle", 3: "csr", 4: "lz4"}
+    traffic = None
+    if os.path.exists(NCU_SUMMARY):
+        with open(NCU_SUMMARY) as f:
+            ncu = json.load(f)
+        k = f"{names[codec]}_{'compress' if d == 0 else 'decompress'}"
+        if k in ncu:
+            traffic = ncu[k].get("dram_bytes_per_algorithmic_byte")
+            traffic = None if traffic is None else round(traffic * g["bytes"] / g["launches"])
+    out = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+           "frac": round(achieved / peak, 4), "traffic": traffic,
+           "kernel": f"{names[codec]}_{'compress' if d == 0 else 'decompress'}", "launches": g["launches"],
+           "algorithmic_bytes_per_launch": g["bytes"] / g["launches"], "avg_launch_ms": g["ms"] / g["launches"],
+           "peak_source": src}
+    out["all_kernels"] = {f"{names[c]}_{'c' if dd == 0 else 'dc'}": {
+        "GBps": round(v["bytes"] / (v["ms"] * 1e-3) / 1e9, 1), "frac": round(v["bytes"] / (v["ms"] * 1e-3) / 1e9 / peak, 4),
+        "ms_total": round(v["ms"], 3), "launches": v["launches"]} for (c, dd), v in groups.items()}
+    return out
+
+
+def _link(torch, nbytes=256 << 20, reps=5) -> dict:
+    host = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    dev = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    res = {}
+    for name, fn in (("d2h", lambda: host.copy_(dev, non_blocking=True)),
+                     ("h2d", lambda: dev.copy_(host, non_blocking=True))):
+        fn()
+        torch.cuda.synchronize()
+        best = 1e9
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            fn()
+            b.record()
+            b.synchronize()
+            best = min(best, a.elapsed_time(b))
+        res[name + "_GBps"] = round(nbytes / (best * 1e-3) / 1e9, 2)
+    return res
+
+
+def _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, raw_bytes, world) -> dict:
+    """Baselines in the same run: vDNN (NONE), SC (always ZVC), the Orac bound; link GB/s;
+    per-tensor latency check (compressed < uncompressed for every tensor the selector compressed)."""
+    ex = {}
+    link = _link(torch)
+    ex["link"] = link
+    steps_b = max(2, min(args.steps, 3))
+    none = timed(C.NONE, steps_b, 1)
+    sc = timed(C.ZVC, steps_b, 1)
+    ex["latency_ms"] = {"auto": main["ms"] / args.steps, "vdnn_none": none["ms"] / steps_b,
+                        "sc_always_zvc": sc["ms"] / steps_b}
+    comp = sum(q["bytes"] for q in main["handles"])
+    orac = comp / (link["d2h_GBps"] * 1e9) + comp / (link["h2d_GBps"] * 1e9)
+    ex["latency_ms"]["orac_bound"] = orac * 1e3
+    ex["latency_ms"]["raw_link_bound"] = (raw_bytes / (link["d2h_GBps"] * 1e9) + raw_bytes / (link["h2d_GBps"] * 1e9)) * 1e3
+    ex["swap_latency_reduction_vs_vdnn"] = 1 - ex["latency_ms"]["auto"] / ex["latency_ms"]["vdnn_none"]
+    # per-tensor: the selector's choice vs NONE, measured one tensor at a time
+    per = []
+    stream = torch.cuda.current_stream()
+    for i, (t, o, n) in enumerate(zip(tensors, outs, sizes)):
+        q = main["handles"][i]
+        row = {"i": i, "MiB": n * w / 2**20, "codec": C.CODEC_NAMES[q["codec"]], "ratio": q["bytes"] / (n * w)}
+        for label, codec in (("none_ms", C.NONE), ("chosen_ms", q["codec"])):
+            best = 1e9
+            for _ in range(3):
+                torch.cuda.synchronize()
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                h = C.swap_out(t, n, dtype, codec)
+                h.swap_in(o)
+                b.record(stream)
+                b.synchronize()
+                h.close()
+                best = min(best, a.elapsed_time(b))
+            row[label] = round(best, 4)
+        per.append(row)
+    ex["per_tensor"] = per
+    ex["every_compressed_tensor_faster"] = all(r["chosen_ms"] < r["none_ms"] for r in per if r["codec"] != "none")
+    return ex
+
+
+def _e2e(args, C, torch, tensors, outs, sizes, dtype, w, dist, world, stream) -> dict:
+    """Same metric through the public API with HOST inputs: per step the 12 inputs are copied
+    H2D from pinned host memory, swapped out and back in, and 16 bytes of every restored
+    tensor are read back D2H."""
+    hosts = [t.cpu().pin_memory() for t in tensors]
+    probe_back = torch.empty(len(tensors), 4, dtype=torch.int32).pin_memory()
+    steps = max(2, min(args.steps, 5))
+
+    def one():
+        for hst, t in zip(hosts, tensors):
+            t.copy_(hst, non_blocking=True)
+        hs = [C.swap_out(t, n, dtype, C.AUTO) for t, n in zip(tensors, sizes)]
+        for o, h in zip(reversed(outs), reversed(hs)):
+            h.swap_in(o)
+        for i, o in enumerate(outs):
+            probe_back[i].copy_(o[:4 * 4 // w].view(torch.int32)[:4], non_blocking=True)
+        return hs
+
+    for h in one():
+        h.close()
+    torch.cuda.synchronize()
+    if dist is not None:
+        dist.barrier()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(stream)
+    for _ in range(steps):
+        for h in one():
+            h.close()
+    b.record(stream)
+    b.synchronize()
+    ms = _max_over_ranks(a.elapsed_time(b), dist) / steps
+    raw = sum(sizes) * w
+    return {"value": round(world * raw / (ms * 1e-3) / 1e9, 3), "unit": "GB/s", "ms_per_step": round(ms, 3),
+            "h2d_bytes_per_step": raw, "d2h_bytes_per_step": 16 * len(tensors), "steps": steps}
+
+
+def _cpu_baseline(tensors, sizes, decisions, dtype, sample_mib=16) -> dict:
+    """The plain-C oracle, as it stands, on the host cores: per tensor the first `sample_mib` MiB
+    are compressed and decompressed with the codec the selector chose (NONE = raw copy)."""
+    import numpy as np
+    from oracle import oracle as O
+    w = 4 if dtype == 0 else 2
+    tot_bytes, tot_s = 0, 0.0
+    for t, n, codec in zip(tensors, sizes, decisions):
+        m = min(n, sample_mib * 2**20 // w)
+        x = t[:m].cpu().numpy()
+        x = x.view(np.uint32) if w == 4 else x.view(np.uint16)
+        t0 = time.perf_counter()
+        blob = O.compress(x, codec, dtype)
+        y = O.decompress(blob, m, dtype)
+        tot_s += time.perf_counter() - t0
+        assert np.array_equal(x, y)
+        tot_bytes += m * w
+    return {"value": round(tot_bytes / tot_s / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+            "sample": f"first {sample_mib} MiB of each of the {len(sizes)} tensors ({tot_bytes / 2**20:.0f} MiB), "
+                      f"oracle compress+decompress with the selector's codec, single thread, {tot_s:.1f} s"}
+
+
+# ------------------------------------------------------------------------------------ reference arm
+def run_reference(args, rank: int, world: int) -> dict | None:
+    """The oracle as it stands on the host cores, same workload / metric / unit: each step is a
+    bounded sample (the first 4 MiB of every tensor of the set): probe + select + compress +
+    decompress on the CPU (there is no link to cross)."""
+    if rank != 0:
+        return None
+    import numpy as np
+
+    import synth
+    from oracle import oracle as O
+    wname, spec, dtype = workload(args.workload)
+    w = synth.WIDTH[dtype]
+    sample = 4 << 20
+    xs = [synth.relu_iid(min(synth.numel(s), sample // w), sp, seed=synth.seed_of(3, 0, 0, i), dtype=dtype)
+          for i, (_, s, sp) in enumerate(spec)]
+    cal = O.make_calib(bw_d2h=50e9, bw_h2d=50e9, alpha_d2h=10e-6, alpha_h2d=10e-6)
+    if os.path.exists(CALIB_PATH):
+        with open(CALIB_PATH) as f:
+            d = json.load(f)["calib"]
+        cal = O.make_calib(alpha_d2h=d["alpha_d2h"], bw_d2h=d["bw_d2h"], alpha_h2d=d["alpha_h2d"],
+                           bw_h2d=d["bw_h2d"], beta=d["beta"], lz4_gamma1=d["lz4_gamma1"],
+                           lz4_gamma2=d["lz4_gamma2"], margin=d["margin"], mode=d["mode"])
+
+    def step():
+        for x in xs:
+            counts = O.probe(x, dtype)
+            codec = O.select(x.size, dtype, counts, 0.0, 0.0, cal)["codec"]
+            blob = O.compress(x, codec, dtype)
+            O.decompress(blob, x.size, dtype)
+
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = (time.perf_counter() - t0) / args.steps
+    nbytes = sum(x.nbytes for x in xs)
+    value = nbytes / dt / 1e9
+    return {"impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32" if w == 4 else "u16", "data": "synthetic",
+            "config": {"workload": wname, "sample": f"first {sample >> 20} MiB of each of {len(xs)} tensors"},
+            "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{nbytes >> 20} MiB per step: probe+select+compress+decompress, 1 thread"},
+            "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="vgg16", choices=["vgg16", "resnet50", "bert"])
+    ap.add_argument("--calibrate", action="store_true", help="full calibration sweep, writes calib/b200.json")
+    ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        res = run_reference(args, rank, world)
+        if res is not None:
+            print(json.dumps(res), flush=True)
+        return
+    dist = None
+    if world > 1:
+        import torch
+        import torch.distributed as tdist
+        torch.cuda.set_device(local_rank)
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        dist = tdist
+    res = run_ours(args, rank, world, local_rank, dist)
+    if rank == 0 and res is not None:
+        print(json.dumps(res), flush=True)
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -171,6 +171,24 @@ cswap_status cswap_fit_time_model(const double* S, const double* s, const double
 /* Ordinary least squares t = alpha + bytes / bw (link model); alpha_out, bw_out. */
 cswap_status cswap_fit_link(const double* bytes, const double* t, uint64_t m, double* alpha_out, double* bw_out);
 
+/* Generic ordinary least squares y = X beta, X row-major m x p (p <= 8); beta_out[p]. */
+cswap_status cswap_fit_linear(const double* X, const double* y, uint64_t m, uint32_t p, double* beta_out);
+
+/* ---- kernel timing (bench / profiling) --------------------------------------------------------- */
+/* One record per timed codec launch group: direction 0 = compress, 1 = decompress, 2 = probe;
+ * raw_bytes = uncompressed bytes covered, comp_bytes = container bytes read or written (0 if
+ * unknown), ms = CUDA-event time on the launch stream. */
+typedef struct {
+  int32_t codec, direction;
+  uint64_t raw_bytes, comp_bytes;
+  double ms;
+} cswap_kernel_record;
+/* When enabled, the swap pipeline brackets its probe / compress / decompress launches with CUDA
+ * events on the stream they are launched on. */
+cswap_status cswap_set_kernel_timing(int enable);
+/* Wait for pending timing events, copy up to `cap` records into `out`, clear; returns the count. */
+uint64_t cswap_collect_kernel_timing(cswap_kernel_record* out, uint64_t cap);
+
 /* ---- diagnostics ---------------------------------------------------------------------------- */
 const char* cswap_status_string(cswap_status s);
 const char* cswap_last_error(void);

@@ -167,6 +167,38 @@ struct Ctx {
   PinnedPool pinned;
   uint32_t* dev_err = nullptr;  // err word for cswap_decompress(err = NULL)
   std::atomic<uint64_t> launches{0};
+  // kernel timing (cswap_set_kernel_timing)
+  std::atomic<bool> timing{false};
+  std::mutex tm_m;
+  struct Pend {
+    cudaEvent_t a, b;
+    cswap_kernel_record r;
+  };
+  std::vector<Pend> pend;
+};
+
+// Brackets a launch group with CUDA events on its stream when timing is enabled.
+struct Timer {
+  Ctx* c;
+  cudaStream_t st;
+  cudaEvent_t a = nullptr, b = nullptr;
+  Timer(Ctx* ctx, cudaStream_t s) : c(ctx), st(s) {
+    if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) cudaEventRecord(a, st);
+  }
+  void stop() {
+    if (a && !b && cudaEventCreate(&b) == cudaSuccess) cudaEventRecord(b, st);
+  }
+  void commit(int codec, int dir, uint64_t raw, uint64_t comp) {
+    if (!a) return;
+    stop();
+    std::lock_guard<std::mutex> lk(c->tm_m);
+    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0}});
+    a = b = nullptr;
+  }
+  ~Timer() {
+    if (a) cudaEventDestroy(a);
+    if (b) cudaEventDestroy(b);
+  }
 };
 
 Ctx* g_ctx = nullptr;
@@ -193,6 +225,7 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
     cudaFree(b.sc.aux);
     cudaFree(b.sc.aux2);
     cudaFree(b.sc.err);
+    cudaFree(b.sc.tbuf);
   }
   tiles = std::max(tiles, b.sc.cap_tiles * 2);
   aux = std::max(aux, b.sc.cap_aux * 2);
@@ -201,6 +234,7 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
   CU(cudaMalloc(&b.sc.aux, aux * 8));
   CU(cudaMalloc(&b.sc.aux2, aux * 8));
   CU(cudaMalloc(&b.sc.err, 64));
+  CU(cudaMalloc(&b.sc.tbuf, tiles * 8));
   CU(cudaMemset(b.sc.status, 0, tiles * 8));
   CU(cudaMemset(b.sc.tickets, 0, kEpochs * 4));
   CU(cudaMemset(b.sc.err, 0, 64));
@@ -239,6 +273,7 @@ struct Lease {
     if (++b->epoch >= kEpochs) {
       cudaMemsetAsync(b->sc.status, 0, b->sc.cap_tiles * 8, st);
       cudaMemsetAsync(b->sc.tickets, 0, kEpochs * 4, st);
+      cudaMemsetAsync(b->sc.aux, 0, b->sc.cap_aux * 8, st);  // epoch-tagged frame starts
       b->epoch = 1;
     }
     return b->epoch;
@@ -319,7 +354,9 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       c->launches++;
       return cuda_status(launch_none_compress(in, n, w, F, dtype, out, out_size, st), "none_compress");
     case CSWAP_CODEC_ZVC: {
-      Lease L(*c, st, zvc_tiles(n, w, F, 0, K, nullptr), K);
+      uint32_t tpf = 0;
+      const uint32_t tiles = zvc_tiles(n, w, F, 0, K, &tpf);
+      Lease L(*c, st, tiles, uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32) + 2);
       TRY(L.status);
       c->launches++;
       return cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, L.b->sc, L.epoch(), dtype, st), "zvc_compress");
@@ -485,6 +522,7 @@ cswap_status cswap_shutdown(void) {
     cudaFree(b.sc.aux);
     cudaFree(b.sc.aux2);
     cudaFree(b.sc.err);
+    cudaFree(b.sc.tbuf);
     cudaEventDestroy(b.ev);
   }
   cudaFree(c->dev_err);
@@ -575,20 +613,29 @@ cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uin
   const cswap_format f = resolve_fmt(c, fmt);
   TRY(check_fmt(f));
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  uint32_t* e = err ? err : c->dev_err;
+  uint32_t* user_err = err ? err : c->dev_err;
   const uint64_t F = f.frame_elems;
   const uint32_t K = uint32_t((n + F - 1) / F);
   Lease L(*c, st, decompress_tiles(n, w, f), decompress_aux(n, w, f));
   TRY(L.status);
+  // kernels flag errors in the lease's device word (never in host-mapped memory: every CTA
+  // reads it); the word is merged into the caller's at the end
+  uint32_t* e = L.b->sc.err;
+  CU(cudaMemsetAsync(e, 0, 4, st));
   const uint8_t* inb = static_cast<const uint8_t*>(in);
-  c->launches++;
+  c->launches += 2;
   TRY(cuda_status(launch_prep(inb, in_size, codec, dtype, n, F, param_of(codec, f), L.b->sc, e, st), "prep"));
-  if (n == 0) return CSWAP_OK;
-  if (codec == CSWAP_CODEC_NONE) {
-    c->launches++;
-    return cuda_status(launch_none_decompress(inb, d_out, n, w, F, L.b->sc, e, st), "none_decompress");
+  cswap_status s = CSWAP_OK;
+  if (n != 0) {
+    if (codec == CSWAP_CODEC_NONE) {
+      c->launches++;
+      s = cuda_status(launch_none_decompress(inb, d_out, n, w, F, L.b->sc, e, st), "none_decompress");
+    } else {
+      s = decompress_range(c, L, inb, d_out, n, dtype, codec, f, 0, K, e, st);
+    }
   }
-  return decompress_range(c, L, inb, d_out, n, dtype, codec, f, 0, K, e, st);
+  TRY(cuda_status(launch_err_merge(e, user_err, st), "err_merge"));
+  return s;
 }
 
 cswap_status cswap_check_device_error(void* stream) {
@@ -623,8 +670,10 @@ static cswap_status probe_impl(Ctx* c, const void* d_in, uint64_t n, int dtype, 
     Lease L(*c, st, 1024, 1024);
     s = L.status;
     if (s == CSWAP_OK) {
+      Timer tm(c, st);
       c->launches++;
       s = cuda_status(launch_probe(d_in, n, w, counts, L.b->sc, L.epoch(), st), "probe");
+      tm.commit(0, 2, std::min<uint64_t>(n, 262144) * w, 0);
     }
     if (s == CSWAP_OK && cudaEventRecord(ev, st) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "event record");
   }
@@ -762,11 +811,14 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     cudaEventDestroy(ready);
     return bail(fail(CSWAP_ERR_NOMEM, "device staging of %llu B failed", (unsigned long long)cap));
   }
+  Timer tm(c, st);
   s = do_compress(c, d_in, n, dtype, use, f, staging, h->size_slot(), st);
+  tm.stop();
   if (s == CSWAP_OK && cudaEventRecord(ready, st) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "event record");
   if (s == CSWAP_OK && cudaEventSynchronize(ready) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "compress failed");
   if (s == CSWAP_OK) {
     h->bytes = *h->size_slot();
+    tm.commit(use, 0, n * uint64_t(w), h->bytes);
     h->host = c->pinned.alloc(h->bytes);
     if (!h->host) s = fail(CSWAP_ERR_NOMEM, "pinned alloc of %llu B failed", (unsigned long long)h->bytes);
   }
@@ -816,6 +868,8 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
   {
     Lease L(*c, st, decompress_tiles(n, w, f), decompress_aux(n, w, f));
     s = L.status;
+    uint32_t* e_dev = L.b->sc.err;  // device word; merged into the handle's pinned slot at the end
+    if (s == CSWAP_OK && cudaMemsetAsync(e_dev, 0, 4, st) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "memset");
     uint64_t off = 0;
     for (uint32_t k0 = 0; k0 < K && s == CSWAP_OK; k0 += fpg) {
       const uint32_t k1 = std::min(K, k0 + fpg);
@@ -833,15 +887,19 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
         s = fail(CSWAP_ERR_CUDA, "prefetch copy failed");
         break;
       }
+      Timer tm(c, st);
       if (k0 == 0) {
         c->launches++;
         s = cuda_status(launch_prep(staging, h->bytes, h->codec, h->dtype, n, F, param_of(h->codec, f), L.b->sc,
-                                    h->err_slot(), st),
+                                    e_dev, st),
                         "prep");
       }
-      if (s == CSWAP_OK) s = decompress_range(c, L, staging, d_out, n, h->dtype, h->codec, f, k0, k1, h->err_slot(), st);
+      if (s == CSWAP_OK) s = decompress_range(c, L, staging, d_out, n, h->dtype, h->codec, f, k0, k1, e_dev, st);
+      const uint64_t raw = (std::min<uint64_t>(n, uint64_t(k1) * F) - uint64_t(k0) * F) * w;
+      tm.commit(h->codec, 1, raw, end - off);
       off = end;
     }
+    if (s == CSWAP_OK) s = cuda_status(launch_err_merge(e_dev, h->err_slot(), st), "err_merge");
   }
   cudaFreeAsync(staging, st);
   cudaEventRecord(h->ev_in, st);
@@ -891,6 +949,41 @@ cswap_status cswap_fit_time_model(const double* S, const double* s, const double
   if (!S || !s || !t || !beta_out) return fail(CSWAP_ERR_INVALID, "NULL argument");
   if (!fit3(S, s, t, m, beta_out)) return fail(CSWAP_ERR_INVALID, "singular or too few samples");
   return CSWAP_OK;
+}
+
+cswap_status cswap_fit_linear(const double* X, const double* y, uint64_t m, uint32_t p, double* beta_out) {
+  if (!X || !y || !beta_out) return fail(CSWAP_ERR_INVALID, "NULL argument");
+  if (!fit_general(X, y, m, p, beta_out)) return fail(CSWAP_ERR_INVALID, "singular, p > 8 or m < p");
+  return CSWAP_OK;
+}
+
+cswap_status cswap_set_kernel_timing(int enable) {
+  Ctx* c = nullptr;
+  TRY(need_ctx(&c));
+  c->timing.store(enable != 0);
+  return CSWAP_OK;
+}
+
+uint64_t cswap_collect_kernel_timing(cswap_kernel_record* out, uint64_t cap) {
+  if (!g_ctx) return 0;
+  Ctx* c = g_ctx;
+  std::vector<Ctx::Pend> p;
+  {
+    std::lock_guard<std::mutex> lk(c->tm_m);
+    p.swap(c->pend);
+  }
+  uint64_t k = 0;
+  for (auto& e : p) {
+    float ms = 0;
+    cudaEventSynchronize(e.b);
+    cudaEventElapsedTime(&ms, e.a, e.b);
+    e.r.ms = ms;
+    if (out && k < cap) out[k] = e.r;
+    k++;
+    cudaEventDestroy(e.a);
+    cudaEventDestroy(e.b);
+  }
+  return std::min(k, cap);
 }
 
 cswap_status cswap_fit_link(const double* bytes, const double* t, uint64_t m, double* alpha_out, double* bw_out) {

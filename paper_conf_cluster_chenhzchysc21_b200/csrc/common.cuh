@@ -33,6 +33,7 @@ struct Scratch {
   uint64_t* aux;          // per-frame / per-block u64 scratch (frame starts, block offsets ...)
   uint64_t* aux2;         // second per-frame / per-tile array
   uint32_t* err;          // device error word (first error wins)
+  uint64_t* tbuf;         // per-tile u64 array for multi-kernel codecs (never epoch-tagged)
   uint64_t cap_tiles, cap_aux;
 };
 
@@ -44,6 +45,16 @@ __device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
 }
 __device__ __forceinline__ void st_release(uint64_t* p, uint64_t v) {
   asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// Polling load: relaxed at gpu scope (no L1 invalidation, unlike ld.acquire which emits
+// CCTL.IVALL).  Status words carry their payload, so relaxed reads are sufficient for them.
+__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ uint32_t ld_acquire32(const uint32_t* p) {
   uint32_t v;
@@ -79,9 +90,10 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* status, int64_t til
     uint64_t s = 0;
     uint32_t f = 0;
     bool ok;
-    do {
+    uint32_t backoff = 32;
+    while (true) {
       if (t >= seg_first) {
-        s = ld_acquire(status + t);
+        s = ld_relaxed(status + t);
         f = status_flag(s, epoch);
         ok = f != 0;
       } else {
@@ -89,7 +101,10 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* status, int64_t til
         f = 0;
         s = 0;
       }
-    } while (!__all_sync(0xffffffffu, ok));
+      if (__all_sync(0xffffffffu, ok)) break;
+      __nanosleep(backoff);
+      backoff = backoff < 512 ? backoff * 2 : 512;
+    }
     const uint32_t pmask = __ballot_sync(0xffffffffu, t >= seg_first && f == kFlagP);
     if (pmask) {
       const int pl = __ffs(pmask) - 1;  // nearest P
@@ -99,6 +114,86 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* status, int64_t til
     }
     uint64_t v = (t >= seg_first) ? status_value(s) : 0;
     excl += warp_sum_u64(v);
+    pos -= 32;
+  }
+}
+
+__device__ __forceinline__ uint64_t warp_suffix_sum_u64(uint64_t v) {  // inclusive, lane l: sum over lanes >= l
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_down_sync(0xffffffffu, v, o);
+    if (lane + o < 32) v += y;
+  }
+  return v;
+}
+
+// Decoupled lookback that also PUBLISHES inclusive prefixes ("P") for the tiles it walks over
+// (up to the last kHist windows before the P it finds).  Tiles later in ticket order then find
+// a P one window back instead of re-walking the same run of aggregates, which keeps the lookback
+// short when hundreds of tiles are in flight.  Publishing is idempotent: any walker computes the
+// same inclusive value for a tile, and only tiles already flagged A are overwritten.
+template <int kHist = 8>
+__device__ __forceinline__ uint64_t lookback_propagate(uint64_t* status, int64_t tile, int64_t seg_first,
+                                                       uint32_t epoch) {
+  const int lane = threadIdx.x & 31;
+  // h[0] = oldest remembered window (closest to `tile`), h[nh-1] = newest; the window in h[k]
+  // covers tiles (pos_P + 32 * (nh - k)) - lane once the P window at pos_P is found.
+  uint64_t h[kHist];
+#pragma unroll
+  for (int k = 0; k < kHist; k++) h[k] = 0;
+  int nh = 0;
+  uint64_t dropped = 0;  // aggregates of windows pushed out of h (closest to `tile`)
+  int64_t pos = tile - 1;
+  while (true) {
+    const int64_t t = pos - lane;
+    const bool inseg = t >= seg_first;
+    uint64_t s = 0;
+    uint32_t f = 0;
+    uint32_t backoff = 32;
+    while (true) {
+      bool ok = true;
+      if (inseg) {
+        s = ld_relaxed(status + t);
+        f = status_flag(s, epoch);
+        ok = f != 0;
+      }
+      if (__all_sync(0xffffffffu, ok)) break;
+      __nanosleep(backoff);
+      backoff = backoff < 512 ? backoff * 2 : 512;
+    }
+    const uint32_t pmask = __ballot_sync(0xffffffffu, inseg && f == kFlagP);
+    if (pmask) {
+      const int pl = __ffs(pmask) - 1;
+      // inclusive value of tile (pos - l), l <= pl: P(pl) + aggregates of lanes l .. pl-1
+      const uint64_t a = lane <= pl ? status_value(s) : 0;
+      const uint64_t incl = warp_suffix_sum_u64(a);
+      if (lane < pl) st_release(status + t, make_status(incl, epoch, kFlagP));
+      uint64_t base = __shfl_sync(0xffffffffu, incl, 0);  // inclusive prefix of tile `pos`
+#pragma unroll
+      for (int k = kHist - 1; k >= 0; k--) {
+        if (k < nh) {
+          const int64_t tp = pos + 32 * (nh - k) - lane;
+          const uint64_t in2 = warp_suffix_sum_u64(h[k]) + base;
+          st_release(status + tp, make_status(in2, epoch, kFlagP));  // these windows are all in-segment
+          base = __shfl_sync(0xffffffffu, in2, 0);
+        }
+      }
+      return base + dropped;
+    }
+    // no P here: remember this window's aggregates (all lanes are in-segment, else a P existed)
+    const uint64_t av = status_value(s);
+    if (nh == kHist) {
+      dropped += warp_sum_u64(h[0]);
+#pragma unroll
+      for (int k = 0; k < kHist - 1; k++) h[k] = h[k + 1];
+      h[kHist - 1] = av;
+    } else {
+#pragma unroll
+      for (int k = 0; k < kHist; k++)
+        if (k == nh) h[k] = av;
+      nh++;
+    }
     pos -= 32;
   }
 }
@@ -131,7 +226,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
       "{\n"
       ".reg .pred p;\n"
       "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 1000000;\n"  // suspend up to 1 ms per try
       "@!p bra WAIT_%=;\n"
       "}\n" ::"r"(a),
       "r"(phase)

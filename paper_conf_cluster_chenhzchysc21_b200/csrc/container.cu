@@ -46,6 +46,17 @@ cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, 
   return cudaGetLastError();
 }
 
+// ---- error word merge (device scratch word -> caller's word, first error wins) ---------------
+__global__ void err_merge_kernel(const uint32_t* src, uint32_t* dst) {
+  const uint32_t v = *src;
+  if (v) atomicCAS(dst, 0u, v);
+}
+
+cudaError_t launch_err_merge(const uint32_t* src, uint32_t* dst, cudaStream_t st) {
+  err_merge_kernel<<<1, 1, 0, st>>>(src, dst);
+  return cudaGetLastError();
+}
+
 // ---- prep: validate the header and scan the frame table --------------------------------------
 __device__ __forceinline__ uint64_t block_excl_scan_u64(uint64_t v, uint64_t* s_warp, uint64_t* total) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;

@@ -12,6 +12,7 @@ cudaError_t launch_header_only(uint8_t* out, int codec, int dtype, uint64_t F, u
                                cudaStream_t st);
 cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
                         uint32_t param, const Scratch& sc, uint32_t* err, cudaStream_t st);
+cudaError_t launch_err_merge(const uint32_t* src, uint32_t* dst, cudaStream_t st);
 cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, int dtype, uint8_t* out,
                                  uint64_t* out_size, cudaStream_t st);
 cudaError_t launch_none_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, const Scratch& sc,

@@ -111,24 +111,21 @@ void decide(uint64_t n, int w, const cswap_probe_result& p, double hf, double hb
   out->codec = best < (1.0 - m) * Tp ? best_c : CSWAP_CODEC_NONE;  // PAPER.md:137, strict
 }
 
-// OLS by modified Gram-Schmidt on column-scaled [1, S, S*s] (robust for S ~ 1e9).
-bool fit3(const double* S, const double* s, const double* t, uint64_t m, double* beta) {
-  if (m < 3) return false;
-  double scale[3] = {1.0, 0.0, 0.0};
-  for (uint64_t i = 0; i < m; i++) {
-    scale[1] = std::fmax(scale[1], std::fabs(S[i]));
-    scale[2] = std::fmax(scale[2], std::fabs(S[i] * s[i]));
+// OLS by modified Gram-Schmidt on column-scaled X (row-major m x p, p <= 8); robust for the
+// badly scaled time-model design [1, S, S*s] with S ~ 1e9.
+bool fit_general(const double* X, const double* y, uint64_t m, uint32_t p, double* beta) {
+  if (p == 0 || p > 8 || m < p) return false;
+  double scale[8];
+  for (uint32_t j = 0; j < p; j++) {
+    scale[j] = 0;
+    for (uint64_t i = 0; i < m; i++) scale[j] = std::fmax(scale[j], std::fabs(X[i * p + j]));
+    if (scale[j] == 0) return false;
   }
-  if (scale[1] == 0) scale[1] = 1;
-  if (scale[2] == 0) scale[2] = 1;
-  std::vector<double> Q(3 * m);
-  for (uint64_t i = 0; i < m; i++) {
-    Q[i] = 1.0;
-    Q[m + i] = S[i] / scale[1];
-    Q[2 * m + i] = S[i] * s[i] / scale[2];
-  }
-  double R[3][3] = {{0}};
-  for (int jc = 0; jc < 3; jc++) {
+  std::vector<double> Q(uint64_t(p) * m);
+  for (uint64_t i = 0; i < m; i++)
+    for (uint32_t j = 0; j < p; j++) Q[j * m + i] = X[i * p + j] / scale[j];
+  double R[8][8] = {{0}};
+  for (int jc = 0; jc < int(p); jc++) {
     double* qj = &Q[jc * m];
     for (int ic = 0; ic < jc; ic++) {
       const double* qi = &Q[ic * m];
@@ -144,20 +141,31 @@ bool fit3(const double* S, const double* s, const double* t, uint64_t m, double*
     if (nrm < 1e-12 * std::sqrt(double(m))) return false;
     for (uint64_t r = 0; r < m; r++) qj[r] /= nrm;
   }
-  double qt[3];
-  for (int jc = 0; jc < 3; jc++) {
+  double qt[8];
+  for (int jc = 0; jc < int(p); jc++) {
     double dot = 0;
-    for (uint64_t r = 0; r < m; r++) dot += Q[jc * m + r] * t[r];
+    for (uint64_t r = 0; r < m; r++) dot += Q[jc * m + r] * y[r];
     qt[jc] = dot;
   }
-  double x[3];
-  for (int jc = 2; jc >= 0; jc--) {
+  double x[8];
+  for (int jc = int(p) - 1; jc >= 0; jc--) {
     double v = qt[jc];
-    for (int kc = jc + 1; kc < 3; kc++) v -= R[jc][kc] * x[kc];
+    for (int kc = jc + 1; kc < int(p); kc++) v -= R[jc][kc] * x[kc];
     x[jc] = v / R[jc][jc];
   }
-  for (int jc = 0; jc < 3; jc++) beta[jc] = x[jc] / scale[jc];
+  for (int jc = 0; jc < int(p); jc++) beta[jc] = x[jc] / scale[jc];
   return true;
+}
+
+// time model of PAPER.md:166: t = b0 + b1*S + b2*S*s
+bool fit3(const double* S, const double* s, const double* t, uint64_t m, double* beta) {
+  std::vector<double> X(3 * m);
+  for (uint64_t i = 0; i < m; i++) {
+    X[3 * i] = 1.0;
+    X[3 * i + 1] = S[i];
+    X[3 * i + 2] = S[i] * s[i];
+  }
+  return fit_general(X.data(), t, m, 3, beta);
 }
 
 bool fit_link(const double* bytes, const double* t, uint64_t m, double* alpha, double* bw) {

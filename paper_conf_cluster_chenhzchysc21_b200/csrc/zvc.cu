@@ -4,19 +4,33 @@
 // additional indexes ... it utilizes a 32-bit bitmap as the index for 32 consecutive floats".
 // Byte layout: DESIGN.md §3 (frame = u32 bitmap[ceil(Fk/32)] pad16 | non-zero words pad16).
 //
-// Compress: ONE pass over the input.  Each CTA takes a 32 KiB tile in ticket order, builds the
-// tile's bitmap words from warp shuffles of per-lane nibbles, counts non-zeros, publishes its
-// byte count (decoupled lookback), learns the absolute container offset of its
-// values, compacts them in shared memory at the destination's 16-byte phase and writes them with
-// 128-bit stores.  Frame k's first tile chains on frame k-1's last tile to place the frame.
-// Decompress: a one-CTA prep kernel validates the header and scans the frame table; then each
-// CTA reads its 1 KiB bitmap slice, popcounts it, gets its in-frame value offset by lookback,
-// pulls its value span into shared memory with one cp.async.bulk (TMA 1-D) and expands it
-// with 128-bit stores.
+// Compress (one pass over the input): a persistent, warp-specialised kernel.
+//   warp 8  (producer): claims 32 KiB tiles in ticket order and streams them into a ring of
+//           shared-memory stages with cp.async.bulk (TMA 1-D) + mbarrier completion;
+//   warps 0-7 (consumers): count tile i+1 (warp ballots -> bitmap words, per-lane ranks) while
+//           the scan warp resolves tile i, then compact tile i at its container offset and store
+//           it with 128-bit stores;
+//   warp 9  (scan): publishes each tile's byte count and resolves its absolute container
+//           offset by decoupled lookback (frame k's first tile chains on frame k-1's end).
+// Decompress (no inter-CTA waiting): tile popcounts of the bitmap (reads n/8 B),
+// a per-frame scan of those counts into value offsets, then one CTA per tile pulls its bitmap
+// slice and value span into shared memory with cp.async.bulk and expands with 128-bit stores.
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <type_traits>
+
 #include "common.cuh"
 #include "kernels.h"
 
 namespace cswap {
+
+// optional phase profiling of the persistent compress kernel (CSWAP_ZVC_PROF=1)
+__device__ unsigned long long g_zprof[16];
+#define ZPROF_ADD(i, v) \
+  do {                  \
+    if (prof) atomicAdd(&g_zprof[i], (unsigned long long)(v)); \
+  } while (0)
 
 template <typename T>
 struct ZvcGeom {
@@ -31,17 +45,14 @@ struct ZvcGeom {
   static_assert(NCH * CHUNK * kWarps == TILE, "tile geometry");
 };
 
-__device__ __forceinline__ uint32_t nib_of(uint4 v, int /*W=4*/, uint32_t /*tag*/) {
-  return (v.x != 0) | ((v.y != 0) << 1) | ((v.z != 0) << 2) | ((v.w != 0) << 3);
-}
-__device__ __forceinline__ uint32_t nib16(uint4 v) {
-  auto h = [](uint32_t u) { return ((u & 0xFFFFu) != 0) | (((u >> 16) != 0) << 1); };
-  return h(v.x) | (h(v.y) << 2) | (h(v.z) << 4) | (h(v.w) << 6);
-}
 template <typename T>
 __device__ __forceinline__ uint32_t nonzero_bits(uint4 v) {
-  if constexpr (sizeof(T) == 4) return nib_of(v, 4, 0);
-  else return nib16(v);
+  if constexpr (sizeof(T) == 4) {
+    return (v.x != 0) | ((v.y != 0) << 1) | ((v.z != 0) << 2) | ((v.w != 0) << 3);
+  } else {
+    auto h = [](uint32_t u) { return ((u & 0xFFFFu) != 0) | (((u >> 16) != 0) << 1); };
+    return h(v.x) | (h(v.y) << 2) | (h(v.z) << 4) | (h(v.w) << 6);
+  }
 }
 template <typename T>
 __device__ __forceinline__ uint32_t lane_elem(const uint4& v, int i) {
@@ -50,349 +61,597 @@ __device__ __forceinline__ uint32_t lane_elem(const uint4& v, int i) {
   else return (w[i >> 1] >> ((i & 1) * 16)) & 0xFFFFu;
 }
 
-// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar)))
+               : "memory");
+}
+__device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
+
+// Read EPV elements starting at tile-relative element e0: from the smem stage where the bulk copy
+// landed, from global memory for the sub-16-byte tail of the tensor, zero past the tile end.
 template <typename T>
-__global__ void __launch_bounds__(kThreads, 4)
-    zvc_compress_kernel(const T* __restrict__ in, uint64_t n, uint64_t F, uint32_t K, uint32_t tpf,
-                        uint32_t num_tiles, uint8_t* __restrict__ out, uint64_t* out_size, Scratch sc,
-                        uint32_t epoch, int dtype) {
+__device__ __forceinline__ uint4 tile_vec(const uint8_t* stage, const T* gsrc, uint32_t e0, uint32_t bulk_elems,
+                                          uint32_t tile_elems) {
   using G = ZvcGeom<T>;
-  __shared__ uint32_t s_ticket;
-  __shared__ uint32_t s_warp_off[kWarps + 1];
-  __shared__ uint64_t s_excl, s_fstart;
-  __shared__ __align__(16) uint32_t s_bm[G::WT];
-  extern __shared__ __align__(16) uint8_t s_out[];  // kTileBytes + 16
+  if (e0 + G::EPV <= bulk_elems) return *reinterpret_cast<const uint4*>(stage + e0 * G::W);
+  uint32_t w4[4] = {0, 0, 0, 0};
+  for (int i = 0; i < G::EPV; i++)
+    if (e0 + i < tile_elems) {
+      const uint32_t x = uint32_t(gsrc[e0 + i]);
+      if constexpr (sizeof(T) == 4) w4[i] = x;
+      else w4[i >> 1] |= x << ((i & 1) * 16);
+    }
+  return make_uint4(w4[0], w4[1], w4[2], w4[3]);
+}
+
+// ------------------------------------------------------------------------------------------
+// compress: persistent, warp-specialised
+//   warp 8  producer: ticket + cp.async.bulk of the tile into stage s          (bar_full[s])
+//   warp 9  resolver: container offset of the tile's values = frame start + bitmap + W x
+//                     (totals of the earlier 32-tile groups of the frame + counts of the
+//                     earlier tiles of its group), all read from published COUNTS  (bar_off[s])
+//   warps 0-7 consumers, per tile: (a) rows of 32 elements -> one ballot = one bitmap word,
+//                     ranks from popcounts (no shuffles); publish the tile count and add it to
+//                     the frame / group accumulators                           (bar_cnt[s]);
+//                     (b) in-place compaction inside the stage (needs no offset); later
+//                     (c) wait for the offset, copy the packed bytes out with 128-bit stores at
+//                     the destination's 16-byte phase, store the bitmap slice, release the
+//                     stage                                                    (bar_empty[s])
+//   The consumers run (a)(b) of tile i+1 before (c) of tile i, so the offset latency overlaps.
+// ------------------------------------------------------------------------------------------
+constexpr int kProducerWarp = kWarps;
+// one resolver warp per stage: a resolver only ever waits on its own stage's barriers, so it can
+// never observe another phase's parity
+template <int S>
+constexpr int compress_threads() { return 32 * (kProducerWarp + 1 + S); }
+
+template <typename T, int S>
+struct CompressSmem {
+  using G = ZvcGeom<T>;
+  static constexpr uint32_t in_off = 0;
+  static constexpr uint32_t bm_off = S * kTileBytes + 128;  // +pad: shifted reads run <= 16 B past a stage
+  static constexpr uint32_t bytes = bm_off + S * G::WT * 4;
+  static constexpr int ctas_per_sm = bytes <= 110 * 1024 ? 2 : 1;
+};
+
+__device__ __forceinline__ uint32_t spread16(uint32_t x) {  // bit i -> bit 2i (i < 16)
+  x &= 0xFFFFu;
+  x = (x | (x << 8)) & 0x00FF00FFu;
+  x = (x | (x << 4)) & 0x0F0F0F0Fu;
+  x = (x | (x << 2)) & 0x33333333u;
+  x = (x | (x << 1)) & 0x55555555u;
+  return x;
+}
+
+template <typename T, int S>
+__global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::ctas_per_sm)
+    zvc_compress_persistent(const T* __restrict__ in, uint64_t n, uint64_t F, uint32_t K, uint32_t tpf,
+                            uint32_t num_tiles, uint8_t* __restrict__ out, uint64_t* out_size, Scratch sc,
+                            uint32_t epoch, int dtype, int prof) {
+  const uint32_t gpf = (tpf + 31) / 32;  // 32-tile groups per frame
+  using G = ZvcGeom<T>;
+  using L = CompressSmem<T, S>;
+  constexpr uint32_t SENT = 0xFFFFFFFFu;
+  constexpr int ROWS = 32;                         // 4-byte loads per lane per tile
+  constexpr int WPR = sizeof(T) == 4 ? 1 : 2;      // bitmap words per row of 32 lanes
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint8_t* s_in = smem + L::in_off;
+  uint32_t* s_bm = reinterpret_cast<uint32_t*>(smem + L::bm_off);  // [S][WT] bitmap words per stage
+  __shared__ __align__(8) uint64_t bar_full[S], bar_empty[S], bar_cnt[S], bar_off[S];
+  __shared__ uint32_t s_ticket[S];
+  __shared__ uint32_t s_nnz[S];
+  __shared__ uint32_t s_wtot[S][kWarps];  // non-zeros per 1024-element slab, per stage
+  __shared__ uint64_t s_off[S], s_fs[S];
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid == 0) s_ticket = atomicAdd(sc.tickets + epoch, 1u);
-  __syncthreads();
-  const uint32_t t = s_ticket;
-  const uint32_t k = t / tpf, j = t % tpf;
-  const uint64_t Fk = frame_len(n, F, k);
-  const uint64_t tin = uint64_t(j) * G::TILE;  // tile start inside the frame
-  const uint32_t tile_elems = uint32_t(umin64(G::TILE, Fk - tin));
-  const T* src = in + uint64_t(k) * F + tin;
-  const bool last_in_frame = tin + G::TILE >= Fk;
-
-  // ---- 1. load, bitmap words, counts ----------------------------------------------------
-  uint4 v[G::NCH];
-  uint32_t bits[G::NCH];
-  uint32_t pos[G::NCH];  // in-warp exclusive rank of this lane's first element, per chunk
-  uint32_t warp_total = 0;
-#pragma unroll
-  for (int q = 0; q < G::NCH; q++) {
-    const uint32_t e0 = warp * G::PER_WARP + q * G::CHUNK + lane * G::EPV;
-    if (e0 + G::EPV <= tile_elems) {
-      v[q] = ldg_stream(reinterpret_cast<const uint4*>(src + e0));
-    } else {
-      uint32_t w4[4] = {0, 0, 0, 0};
-      for (int i = 0; i < G::EPV; i++)
-        if (e0 + i < tile_elems) {
-          uint32_t x = uint32_t(src[e0 + i]);
-          if constexpr (sizeof(T) == 4) w4[i] = x;
-          else w4[i >> 1] |= x << ((i & 1) * 16);
-        }
-      v[q] = make_uint4(w4[0], w4[1], w4[2], w4[3]);
-    }
-  }
-#pragma unroll
-  for (int q = 0; q < G::NCH; q++) {
-    const uint32_t b = nonzero_bits<T>(v[q]);
-    bits[q] = b;
-    // bitmap word = OR of the LPW lanes' bit groups, each shifted to its element position
-    uint32_t word = b << ((lane % G::LPW) * G::EPV);
-    word |= __shfl_xor_sync(0xffffffffu, word, 1);
-    word |= __shfl_xor_sync(0xffffffffu, word, 2);
-    if (G::LPW >= 8) word |= __shfl_xor_sync(0xffffffffu, word, 4);
-    if (lane % G::LPW == 0) s_bm[(warp * G::PER_WARP + q * G::CHUNK) / 32 + lane / G::LPW] = word;
-    // inclusive warp scan of per-lane counts
-    const uint32_t c = __popc(b);
-    uint32_t inc = c;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
-      if (lane >= o) inc += y;
-    }
-    pos[q] = warp_total + inc - c;
-    warp_total += __shfl_sync(0xffffffffu, inc, 31);
-  }
-  if (lane == 0) s_warp_off[warp + 1] = warp_total;
-  __syncthreads();
   if (tid == 0) {
-    uint32_t acc = 0;
-    s_warp_off[0] = 0;
-    for (int w = 0; w < kWarps; w++) {
-      acc += s_warp_off[w + 1];
-      s_warp_off[w + 1] = acc;
+    for (int s = 0; s < S; s++) {
+      mbar_init(&bar_full[s], 1);
+      mbar_init(&bar_empty[s], kWarps);
+      mbar_init(&bar_cnt[s], 1);
+      mbar_init(&bar_off[s], 1);
     }
   }
   __syncthreads();
-  const uint32_t tile_nnz = s_warp_off[kWarps];
-  const uint64_t tile_bytes = uint64_t(tile_nnz) * G::W;
 
-  // ---- 2. publish aggregate, look back, publish inclusive prefix --------------------------
-  const uint64_t nwords_k = cdiv(Fk, 32);
-  if (warp == 0) {
-    if (j > 0 && lane == 0) st_release(sc.status + t, make_status(tile_bytes, epoch, kFlagA));
-    uint64_t excl, fstart;
-    if (j == 0) {
+  auto tile_geom = [&](uint32_t t, uint32_t& k, uint32_t& j, uint64_t& Fk, uint32_t& tile_elems,
+                       uint32_t& bulk_elems) {
+    k = t / tpf;
+    j = t % tpf;
+    Fk = frame_len(n, F, k);
+    tile_elems = uint32_t(umin64(G::TILE, Fk - uint64_t(j) * G::TILE));
+    bulk_elems = ((tile_elems * G::W) & ~15u) / G::W;
+  };
+
+  if (warp == kProducerWarp) {  // ----------------------------------------- producer (TMA)
+    for (uint32_t i = 0;; i++) {
+      const int s = i % S;
+      long long c0 = clock64();
+      if (i >= S) mbar_wait(&bar_empty[s], ((i / S) - 1) & 1);
+      if (lane == 0) ZPROF_ADD(0, clock64() - c0);
+      uint32_t t = 0;
+      if (lane == 0) t = atomicAdd(sc.tickets + epoch, 1u);
+      t = __shfl_sync(0xffffffffu, t, 0);
+      if (t >= num_tiles) {
+        if (lane == 0) {
+          s_ticket[s] = SENT;
+          mbar_arrive(&bar_full[s]);
+        }
+        break;
+      }
       if (lane == 0) {
+        uint32_t k, j, te, be;
+        uint64_t Fk;
+        tile_geom(t, k, j, Fk, te, be);
+        s_ticket[s] = t;
+        if (be) {
+          mbar_expect_tx(&bar_full[s], be * G::W);
+          bulk_g2s(s_in + s * kTileBytes, in + uint64_t(k) * F + uint64_t(j) * G::TILE, be * G::W, &bar_full[s]);
+        } else {
+          mbar_arrive(&bar_full[s]);
+        }
+      }
+    }
+    return;
+  }
+
+  if (warp > kProducerWarp) {  // -------------------------------- resolvers (one per stage)
+    const int r = warp - kProducerWarp - 1;
+    for (uint32_t i = r;; i += S) {
+      const int s = r;
+      long long c0 = clock64();
+      mbar_wait(&bar_cnt[s], (i / S) & 1);
+      long long c1 = clock64();
+      if (lane == 0) ZPROF_ADD(2, c1 - c0);
+      const uint32_t nnz = s_nnz[s];
+      if (nnz == SENT) break;
+      const uint32_t t = s_ticket[s];
+      const uint32_t k = t / tpf, j = t % tpf;
+      const uint64_t nwords_k = cdiv(frame_len(n, F, k), 32);
+      uint64_t excl = 0, fstart = 0;
+      // offset = frame start + bitmap + W * (totals of earlier 32-tile groups of the frame +
+      // counts of earlier tiles of the group).  Everything comes from COUNTS (published as soon
+      // as a tile lands), never from other tiles' resolutions, so no chain forms across tiles.
+      if (j == 0 && lane == 0) {
         if (k == 0) {
           fstart = data_start(K);
-        } else {
-          uint64_t s;
-          do { s = ld_acquire(sc.status + t - 1); } while (status_flag(s, epoch) != kFlagP);
-          fstart = a16(status_value(s));
+        } else {  // previous frame's start + its bitmap + its packed values (from its accumulator)
+          uint64_t a, acc;
+          uint32_t backoff = 32;
+          while (status_flag(a = ld_relaxed(sc.aux + k - 1), epoch) != kFlagP) {
+            __nanosleep(backoff);
+            backoff = backoff < 256 ? backoff * 2 : 256;
+          }
+          const uint64_t Fp = frame_len(n, F, k - 1);
+          const uint64_t tiles_prev = cdiv(Fp, G::TILE);
+          backoff = 32;
+          while (((acc = ld_relaxed(sc.aux2 + k - 1)) >> 40) != tiles_prev) {
+            __nanosleep(backoff);
+            backoff = backoff < 256 ? backoff * 2 : 256;
+          }
+          fstart = status_value(a) + a16(4 * cdiv(Fp, 32)) + a16(G::W * (acc & ((1ull << 40) - 1)));
         }
-        excl = fstart + a16(4 * nwords_k);
-        st_release(sc.aux + k, fstart);
-        st_release(sc.status + t, make_status(excl + tile_bytes, epoch, kFlagP));
-        s_excl = excl;
-        s_fstart = fstart;
+        st_relaxed(sc.aux + k, make_status(fstart, epoch, kFlagP));
       }
-    } else {
-      excl = lookback(sc.status, t, int64_t(t) - j, epoch);
+      uint64_t prefix = 0;  // non-zeros of the frame before this tile
+      {
+        const uint32_t g = j / 32;
+        for (uint32_t g0 = 0; g0 < g; g0 += 32) {  // complete groups before g (32 tiles each)
+          const uint32_t gi = g0 + lane;
+          uint64_t v = 0;
+          if (gi < g) {
+            const uint64_t* p = sc.aux2 + K + uint64_t(k) * gpf + gi;
+            uint32_t backoff = 32;
+            while (((v = ld_relaxed(p)) >> 40) != 32) {
+              __nanosleep(backoff);
+              backoff = backoff < 256 ? backoff * 2 : 256;
+            }
+            v &= (1ull << 40) - 1;
+          }
+          prefix += warp_sum_u64(v);
+        }
+        const uint32_t jj = j - 32 * g;  // earlier tiles of this group
+        uint64_t v = 0;
+        if (uint32_t(lane) < jj) {
+          const uint64_t* p = sc.status + (t - jj + lane);
+          uint64_t st;
+          uint32_t backoff = 32;
+          while (status_flag(st = ld_relaxed(p), epoch) == 0) {
+            __nanosleep(backoff);
+            backoff = backoff < 256 ? backoff * 2 : 256;
+          }
+          v = status_value(st);
+        }
+        prefix += warp_sum_u64(v);
+      }
       if (lane == 0) {
-        st_release(sc.status + t, make_status(excl + tile_bytes, epoch, kFlagP));
-        s_excl = excl;
-        s_fstart = ld_acquire(sc.aux + k);
+        if (j != 0) {
+          uint64_t a;
+          uint32_t backoff = 32;
+          while (status_flag(a = ld_relaxed(sc.aux + k), epoch) != kFlagP) {
+            __nanosleep(backoff);
+            backoff = backoff < 256 ? backoff * 2 : 256;
+          }
+          fstart = status_value(a);
+        }
+        excl = fstart + a16(4 * nwords_k) + uint64_t(G::W) * prefix;
       }
+      if (lane == 0) {
+        ZPROF_ADD(3, clock64() - c1);
+        s_off[s] = excl;
+        s_fs[s] = fstart;
+        mbar_arrive(&bar_off[s]);
+      }
+      __syncwarp();
     }
+    return;
   }
-  __syncthreads();
-  const uint64_t g0 = s_excl, fstart = s_fstart;
-  const uint32_t d = uint32_t(g0 & 15);
 
-  // ---- 3. compact into shared memory at the destination's 16-byte phase ------------------
-  const uint32_t woff = s_warp_off[warp];
-#pragma unroll
-  for (int q = 0; q < G::NCH; q++) {
-    uint32_t b = bits[q];
-    uint32_t r = woff + pos[q];
-#pragma unroll
-    for (int i = 0; i < G::EPV; i++) {
-      if (b & (1u << i)) {
-        const uint32_t x = lane_elem<T>(v[q], i);
-        if constexpr (sizeof(T) == 4) *reinterpret_cast<uint32_t*>(s_out + d + 4 * r) = x;
-        else *reinterpret_cast<uint16_t*>(s_out + d + 2 * r) = uint16_t(x);
-        r++;
-      }
-    }
-  }
-  __syncthreads();
+  // ------------------------------------------------------------------------- consumers
+  // 8 warps, warp w owns slab w (1024 elements = 32 rows of 32 four-byte words) of every tile.
+  // count(i):   rows -> one ballot per row = one bitmap word (fp32) / two ballots (16-bit);
+  //             slab totals; the tile count is published (A) and added to the accumulators.
+  // emit(i-1):  wait for tile i-1's offset, re-read its rows from the stage and store every
+  //             non-zero straight to global memory at its rank (a warp's predicated 4-byte
+  //             stores of one row cover a contiguous range); store the slab's bitmap words.
+  // count(i) runs before emit(i-1), so a tile's count never waits for an older tile's offset.
+  const uint32_t lt = (1u << lane) - 1u;
+  constexpr uint32_t SLAB = G::PER_WARP * G::W;  // bytes per slab (4 KiB)
+  auto load_row = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t q, uint32_t te, uint32_t be) {
+    constexpr bool full = decltype(full_tag)::value;
+    if (full) return reinterpret_cast<const uint32_t*>(stage)[q];
+    if (sizeof(T) == 4) return q < be ? reinterpret_cast<const uint32_t*>(stage)[q] : (q < te ? uint32_t(gsrc[q]) : 0u);
+    const uint32_t e = 2 * q;
+    if (e + 2 <= be) return reinterpret_cast<const uint32_t*>(stage)[q];
+    return (e < te ? uint32_t(gsrc[e]) : 0u) | ((e + 1 < te ? uint32_t(gsrc[e + 1]) : 0u) << 16);
+  };
+  auto group_wait = [&](uint64_t* bar, uint32_t parity) {  // one warp polls, the rest block in bar.sync
+    if (warp == 0) mbar_wait(bar, parity);
+    consumer_sync();
+    if (warp != 0) mbar_wait(bar, parity);  // phase already complete: returns at once
+  };
 
-  // ---- 4. stores: values (16-byte vectors, element-wise head/tail), bitmap, frame pad -----
-  uint8_t* gdst = out + (g0 - d);
-  const uint32_t span = d + uint32_t(tile_bytes);
-  const uint32_t nvec = (span + 15) / 16;
-  for (uint32_t c = tid; c < nvec; c += kThreads) {
-    const uint32_t lo = 16 * c, hi = lo + 16;
-    if (lo >= d && hi <= span) {
-      stg_stream(reinterpret_cast<uint4*>(gdst + lo), *reinterpret_cast<const uint4*>(s_out + lo));
-    } else {
-      for (uint32_t b = max(lo, d); b < min(hi, span); b += G::W) {
-        if constexpr (sizeof(T) == 4) *reinterpret_cast<uint32_t*>(gdst + b) = *reinterpret_cast<const uint32_t*>(s_out + b);
-        else *reinterpret_cast<uint16_t*>(gdst + b) = *reinterpret_cast<const uint16_t*>(s_out + b);
+  auto count_slab = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be,
+                        uint32_t* bm_out) {
+    const uint32_t q0 = warp * (SLAB / 4);
+    uint32_t tot = 0;
+#pragma unroll 8
+    for (int m = 0; m < ROWS; m++) {
+      const uint32_t v = load_row(full_tag, stage, gsrc, q0 + 32 * m + lane, te, be);
+      if (sizeof(T) == 4) {
+        const uint32_t w = __ballot_sync(0xffffffffu, v != 0);
+        if (lane == 0) bm_out[m] = w;
+        tot += __popc(w);
+      } else {
+        const uint32_t lo = __ballot_sync(0xffffffffu, (v & 0xFFFFu) != 0);
+        const uint32_t hi = __ballot_sync(0xffffffffu, (v >> 16) != 0);
+        if (lane == 0) {
+          bm_out[2 * m] = spread16(lo) | (spread16(hi) << 1);
+          bm_out[2 * m + 1] = spread16(lo >> 16) | (spread16(hi >> 16) << 1);
+        }
+        tot += __popc(lo) + __popc(hi);
       }
     }
-  }
-  const uint64_t g1 = g0 + tile_bytes;
-  if (last_in_frame && tid == kThreads - 1) {
-    for (uint64_t b = g1; b < a16(g1); b += 2) *reinterpret_cast<uint16_t*>(out + b) = 0;
-    *reinterpret_cast<uint64_t*>(out + 64 + 8ull * k) = a16(g1) - fstart;  // frame_bytes[k]
-  }
-  {
-    const uint64_t w0 = uint64_t(j) * G::WT;
-    const uint64_t wend = last_in_frame ? ((nwords_k + 3) & ~uint64_t(3)) : w0 + G::WT;
-    const uint32_t nv = uint32_t((wend - w0) / 4);
-    uint4* bdst = reinterpret_cast<uint4*>(out + fstart + 4 * w0);
-    for (uint32_t c = tid; c < nv; c += kThreads) stg_stream(bdst + c, reinterpret_cast<const uint4*>(s_bm)[c]);
-  }
-  if (t == num_tiles - 1 && tid == 0) {
-    const uint64_t total = a16(g1);
-    write_header(out, kZVC, dtype, n, F, K, 0, total);
-    for (uint64_t b = 64 + 8ull * K; b < data_start(K); b += 8) *reinterpret_cast<uint64_t*>(out + b) = 0;
-    *out_size = total;
+    return tot;
+  };
+
+  auto emit_slab = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be, uint8_t* dst) {
+    const uint32_t q0 = warp * (SLAB / 4);
+    uint32_t pre = 0;
+#pragma unroll 8
+    for (int m = 0; m < ROWS; m++) {
+      const uint32_t v = load_row(full_tag, stage, gsrc, q0 + 32 * m + lane, te, be);
+      if (sizeof(T) == 4) {
+        const uint32_t w = __ballot_sync(0xffffffffu, v != 0);
+        if (v) reinterpret_cast<uint32_t*>(dst)[pre + __popc(w & lt)] = v;
+        pre += __popc(w);
+      } else {
+        const uint32_t lo = __ballot_sync(0xffffffffu, (v & 0xFFFFu) != 0);
+        const uint32_t hi = __ballot_sync(0xffffffffu, (v >> 16) != 0);
+        uint32_t r = pre + __popc(lo & lt) + __popc(hi & lt);
+        uint16_t* d16 = reinterpret_cast<uint16_t*>(dst);
+        if (v & 0xFFFFu) d16[r++] = uint16_t(v);
+        if (v >> 16) d16[r] = uint16_t(v >> 16);
+        pre += __popc(lo) + __popc(hi);
+      }
+    }
+  };
+
+  auto count = [&](uint32_t i, uint32_t t) {
+    const int s = i % S;
+    uint32_t k, j, te, be;
+    uint64_t Fk;
+    tile_geom(t, k, j, Fk, te, be);
+    const T* gsrc = in + uint64_t(k) * F + uint64_t(j) * G::TILE;
+    const uint8_t* stage = s_in + s * kTileBytes;
+    uint32_t* bm_out = s_bm + s * G::WT + warp * (G::WT / kWarps);
+    const uint32_t c = (te == G::TILE && be == G::TILE) ? count_slab(std::true_type{}, stage, gsrc, te, be, bm_out)
+                                                        : count_slab(std::false_type{}, stage, gsrc, te, be, bm_out);
+    if (lane == 0) s_wtot[s][warp] = c;
+    consumer_sync();
+    if (tid == 0) {  // publish the tile count (A) and feed the frame / group accumulators
+      uint32_t tot = 0;
+#pragma unroll
+      for (int w = 0; w < kWarps; w++) tot += s_wtot[s][w];
+      st_relaxed(sc.status + t, make_status(tot, epoch, kFlagA));  // self-contained: no release needed
+      atomicAdd(reinterpret_cast<unsigned long long*>(sc.aux2 + k), (1ull << 40) + tot);
+      atomicAdd(reinterpret_cast<unsigned long long*>(sc.aux2 + K + uint64_t(k) * gpf + j / 32), (1ull << 40) + tot);
+      s_nnz[s] = tot;
+      mbar_arrive(&bar_cnt[s]);
+    }
+  };
+
+  auto emit = [&](uint32_t i, uint32_t t) {
+    const int s = i % S;
+    long long c0 = clock64();
+    group_wait(&bar_off[s], (i / S) & 1);
+    if (tid == 0) ZPROF_ADD(5, clock64() - c0);
+    long long c2 = clock64();
+    const uint64_t g0 = s_off[s], fstart = s_fs[s];
+    uint32_t k, j, te, be;
+    uint64_t Fk;
+    tile_geom(t, k, j, Fk, te, be);
+    const T* gsrc = in + uint64_t(k) * F + uint64_t(j) * G::TILE;
+    const uint8_t* stage = s_in + s * kTileBytes;
+    uint32_t woff = 0, nnz = 0;
+#pragma unroll
+    for (int w = 0; w < kWarps; w++) {
+      const uint32_t x = s_wtot[s][w];
+      woff += w < warp ? x : 0;
+      nnz += x;
+    }
+    uint8_t* dst = out + g0 + uint64_t(G::W) * woff;
+    if (te == G::TILE && be == G::TILE) emit_slab(std::true_type{}, stage, gsrc, te, be, dst);
+    else emit_slab(std::false_type{}, stage, gsrc, te, be, dst);
+    {  // this slab's bitmap words, clipped to the frame's bitmap section (incl. its 16-byte pad)
+      constexpr uint32_t WPW = G::WT / kWarps;
+      const uint64_t wsec = (cdiv(Fk, 32) + 3) & ~uint64_t(3);
+      const uint64_t w0 = uint64_t(j) * G::WT + warp * WPW;
+      if (w0 < wsec) {
+        const uint32_t nv = uint32_t((umin64(w0 + WPW, wsec) - w0) / 4);
+        uint4* bdst = reinterpret_cast<uint4*>(out + fstart + 4 * w0);
+        const uint4* bsrc = reinterpret_cast<const uint4*>(s_bm + s * G::WT + warp * WPW);
+        if (uint32_t(lane) < nv) stg_stream(bdst + lane, bsrc[lane]);
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&bar_empty[s]);  // this warp no longer reads the stage
+    const uint64_t g1 = g0 + uint64_t(nnz) * G::W;
+    if (warp == kWarps - 1 && lane == 31) {
+      if (uint64_t(j) * G::TILE + G::TILE >= Fk) {  // last tile of the frame: pad + frame_bytes[k]
+        for (uint64_t b = g1; b < a16(g1); b += 2) *reinterpret_cast<uint16_t*>(out + b) = 0;
+        *reinterpret_cast<uint64_t*>(out + 64 + 8ull * k) = a16(g1) - fstart;
+      }
+      if (t == num_tiles - 1) {
+        const uint64_t total = a16(g1);
+        write_header(out, kZVC, dtype, n, F, K, 0, total);
+        for (uint64_t b = 64 + 8ull * K; b < data_start(K); b += 8) *reinterpret_cast<uint64_t*>(out + b) = 0;
+        *out_size = total;
+      }
+    }
+    if (tid == 0) ZPROF_ADD(6, clock64() - c2);
+  };
+
+  uint32_t prev_t = SENT;
+  for (uint32_t i = 0;; i++) {
+    const int s = i % S;
+    long long c0 = clock64();
+    group_wait(&bar_full[s], (i / S) & 1);
+    if (tid == 0) ZPROF_ADD(7, clock64() - c0);
+    const uint32_t t = s_ticket[s];
+    if (t == SENT) {
+      if (tid == 0) {  // no more work: tell every resolver
+        for (uint32_t i2 = i; i2 < i + S; i2++) {
+          s_nnz[i2 % S] = SENT;
+          mbar_arrive(&bar_cnt[i2 % S]);
+        }
+      }
+      if (prev_t != SENT) emit(i - 1, prev_t);
+      break;
+    }
+    long long c3 = clock64();
+    count(i, t);
+    if (tid == 0) ZPROF_ADD(8, clock64() - c3);
+    if (prev_t != SENT) emit(i - 1, prev_t);
+    prev_t = t;
   }
 }
 
 // ------------------------------------------------------------------------------------------
+// decompress: counts -> per-frame scan -> expand
+// ------------------------------------------------------------------------------------------
+// One warp per tile: popcount of the tile's bitmap slice; checks the bits past the frame end.
 template <typename T>
-__global__ void __launch_bounds__(kThreads, 4)
-    zvc_decompress_kernel(const uint8_t* __restrict__ in, T* __restrict__ outp, uint64_t n, uint64_t F,
-                          uint32_t K, uint32_t tpf, uint32_t k0, uint32_t num_tiles, Scratch sc, uint32_t epoch,
-                          uint32_t* err) {
+__global__ void __launch_bounds__(kThreads) zvc_count_kernel(const uint8_t* __restrict__ in, uint64_t n, uint64_t F,
+                                                             uint32_t tpf, uint32_t k0, uint32_t num_tiles,
+                                                             Scratch sc, uint32_t* err) {
   using G = ZvcGeom<T>;
-  __shared__ uint32_t s_ticket;
-  __shared__ uint32_t s_warp_off[kWarps + 1];
-  __shared__ uint64_t s_excl;
-  __shared__ __align__(8) uint64_t s_bar;
-  __shared__ __align__(16) uint32_t s_bm[G::WT];
-  extern __shared__ __align__(16) uint8_t s_val[];  // kTileBytes + 32
-
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (*reinterpret_cast<volatile uint32_t*>(err) != 0) return;  // header rejected by prep
-  if (tid == 0) s_ticket = atomicAdd(sc.tickets + epoch, 1u);
-  __syncthreads();
-  const uint32_t t = s_ticket + k0 * tpf;  // status index (frame-major)
+  const int lane = threadIdx.x & 31;
+  const uint32_t tl = blockIdx.x * kWarps + (threadIdx.x >> 5);
+  if (tl >= num_tiles || *reinterpret_cast<volatile const uint32_t*>(err)) return;
+  const uint32_t t = tl + k0 * tpf;
   const uint32_t k = t / tpf, j = t % tpf;
   const uint64_t Fk = frame_len(n, F, k);
-  const uint64_t tin = uint64_t(j) * G::TILE;
-  const uint32_t tile_elems = uint32_t(umin64(G::TILE, Fk - tin));
-  const uint64_t fstart = sc.aux[k];
-  const uint64_t fbytes = sc.aux2[k];
-  const uint64_t nwords_k = cdiv(Fk, 32);
-  const uint64_t bm_bytes = a16(4 * nwords_k);
-  const bool last_in_frame = tin + G::TILE >= Fk;
-  bool bad = bm_bytes > fbytes;
-
-  // ---- 1. bitmap slice -> smem; counts ---------------------------------------------------
-  const uint32_t nw_tile = uint32_t(cdiv(tile_elems, 32));
-  {
-    const uint32_t* bsrc = reinterpret_cast<const uint32_t*>(in + fstart) + uint64_t(j) * G::WT;
-    const uint32_t nv = (nw_tile + 3) / 4;
-    for (uint32_t c = tid; c < G::WT / 4; c += kThreads) {
-      uint4 x = make_uint4(0, 0, 0, 0);
-      if (c < nv && !bad) x = *reinterpret_cast<const uint4*>(bsrc + 4 * c);
-      reinterpret_cast<uint4*>(s_bm)[c] = x;
+  const uint32_t tile_elems = uint32_t(umin64(G::TILE, Fk - uint64_t(j) * G::TILE));
+  const uint32_t nw = (tile_elems + 31) / 32;
+  const uint64_t fstart = sc.aux[k], fbytes = sc.aux2[k];
+  if (a16(4 * cdiv(Fk, 32)) > fbytes) {
+    if (lane == 0) set_error(err, kErrCorrupt);
+    return;
+  }
+  const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + fstart) + uint64_t(j) * G::WT;
+  uint32_t c = 0;
+  for (uint32_t w = lane; w < nw; w += 32) {
+    uint32_t x = bm[w];
+    if (w == nw - 1 && (tile_elems & 31)) {
+      const uint32_t keep = (1u << (tile_elems & 31)) - 1;
+      if (x & ~keep) set_error(err, kErrCorrupt);
+      x &= keep;
     }
+    c += __popc(x);
   }
-  if (tid == 0) mbar_init(&s_bar, 1);
-  __syncthreads();
-  if (tid == 0 && (tile_elems & 31)) {  // bits past the frame end must be zero
-    uint32_t& last = s_bm[nw_tile - 1];
-    if (last >> (tile_elems & 31)) { bad = true; last &= (1u << (tile_elems & 31)) - 1; }
-  }
-  if (bad) set_error(err, kErrCorrupt);
-  __syncthreads();
-  uint32_t wt = 0;
-  {
-    constexpr int WPW = G::WT / kWarps;  // words per warp (32 or 64)
+  c = __reduce_add_sync(0xffffffffu, c);
+  if (lane == 0) sc.tbuf[t] = c;
+}
+
+// One CTA per frame: exclusive scan of tile counts -> absolute value offsets; validates the
+// frame size against the header's frame table.
+template <typename T>
+__global__ void __launch_bounds__(1024) zvc_scan_kernel(uint64_t n, uint64_t F, uint32_t tpf, uint32_t k0, Scratch sc,
+                                                        uint32_t* err) {
+  using G = ZvcGeom<T>;
+  __shared__ uint64_t s_w[33];
+  if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
+  const uint32_t k = k0 + blockIdx.x;
+  const uint64_t Fk = frame_len(n, F, k);
+  const uint32_t nt = uint32_t(cdiv(Fk, G::TILE));
+  const uint64_t base = sc.aux[k] + a16(4 * cdiv(Fk, 32));
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t carry = 0;
+  for (uint32_t c0 = 0; c0 < nt; c0 += blockDim.x) {
+    const uint32_t j = c0 + threadIdx.x;
+    const uint64_t v = j < nt ? sc.tbuf[uint64_t(k) * tpf + j] : 0;
+    uint64_t inc = v;
 #pragma unroll
-    for (int i = 0; i < WPW / 32; i++) wt += __popc(s_bm[warp * WPW + i * 32 + lane]);
-    wt = __reduce_add_sync(0xffffffffu, wt);
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += y;
+    }
+    if (lane == 31) s_w[warp] = inc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint64_t acc = 0;
+      for (int w = 0; w < int(blockDim.x / 32); w++) {
+        const uint64_t x = s_w[w];
+        s_w[w] = acc;
+        acc += x;
+      }
+      s_w[32] = acc;
+    }
+    __syncthreads();
+    if (j < nt) sc.tbuf[uint64_t(k) * tpf + j] = base + G::W * (carry + s_w[warp] + inc - v);
+    carry += s_w[32];
+    __syncthreads();
   }
-  if (lane == 0) s_warp_off[warp + 1] = wt;
-  __syncthreads();
+  if (threadIdx.x == 0 && a16(4 * cdiv(Fk, 32)) + a16(G::W * carry) != sc.aux2[k]) set_error(err, kErrCorrupt);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kThreads) zvc_expand_kernel(const uint8_t* __restrict__ in, T* __restrict__ outp,
+                                                              uint64_t n, uint64_t F, uint32_t tpf, uint32_t k0,
+                                                              Scratch sc, uint32_t* err) {
+  using G = ZvcGeom<T>;
+  __shared__ __align__(8) uint64_t s_bar;
+  __shared__ __align__(16) uint32_t s_bm[G::WT + 4];
+  __shared__ uint32_t s_woff[kWarps];
+  extern __shared__ __align__(16) uint8_t s_val[];  // kTileBytes + 32
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
+  const uint32_t t = blockIdx.x + k0 * tpf;
+  const uint32_t k = t / tpf, j = t % tpf;
+  const uint64_t Fk = frame_len(n, F, k);
+  const uint32_t tile_elems = uint32_t(umin64(G::TILE, Fk - uint64_t(j) * G::TILE));
+  const uint32_t nw = (tile_elems + 31) / 32;
+  const uint64_t fstart = sc.aux[k], fend = fstart + sc.aux2[k];
+  const uint64_t vbeg = sc.tbuf[t];
+  const uint64_t vend = (j + 1 < uint32_t(cdiv(Fk, G::TILE))) ? sc.tbuf[t + 1] : 0;  // next tile's start
   if (tid == 0) {
-    uint32_t acc = 0;
-    s_warp_off[0] = 0;
-    for (int w = 0; w < kWarps; w++) {
-      acc += s_warp_off[w + 1];
-      s_warp_off[w + 1] = acc;
-    }
+    mbar_init(&s_bar, 1);
   }
   __syncthreads();
-  const uint32_t tile_nnz = s_warp_off[kWarps];
-
-  // ---- 2. in-frame popcount prefix by lookback ------------------------------------------
-  if (warp == 0) {
-    uint64_t excl = 0;
-    if (j > 0) {
-      if (lane == 0) st_release(sc.status + t, make_status(tile_nnz, epoch, kFlagA));
-      excl = lookback(sc.status, t, int64_t(t) - j, epoch);
+  // tile value count = popcount of the bitmap slice; the span end for the last tile of the
+  // frame comes from the count, for others from the next tile's offset
+  const uint32_t bm_bytes = ((nw * 4) + 15) & ~15u;
+  const uint8_t* bsrc = in + fstart + uint64_t(j) * G::WT * 4;
+  if (tid == 0) {
+    mbar_expect_tx(&s_bar, bm_bytes);
+    bulk_g2s(s_bm, bsrc, bm_bytes, &s_bar);
+  }
+  mbar_wait(&s_bar, 0);
+  // per-warp totals
+  {
+    constexpr int WPW = G::WT / kWarps;
+    uint32_t c = 0;
+#pragma unroll
+    for (int i = 0; i < WPW / 32; i++) {
+      const uint32_t wi = warp * WPW + i * 32 + lane;
+      uint32_t x = wi < nw ? s_bm[wi] : 0;
+      if (wi == nw - 1 && (tile_elems & 31)) x &= (1u << (tile_elems & 31)) - 1;
+      c += __popc(x);
     }
-    if (lane == 0) {
-      st_release(sc.status + t, make_status(excl + tile_nnz, epoch, kFlagP));
-      s_excl = excl;
-      if (last_in_frame && bm_bytes + a16(G::W * (excl + tile_nnz)) != fbytes) set_error(err, kErrCorrupt);
-    }
+    c = __reduce_add_sync(0xffffffffu, c);
+    if (lane == 0) s_woff[warp] = c;
   }
   __syncthreads();
-  const uint64_t excl = s_excl;
-
-  // ---- 3. value span -> smem with one bulk copy (aligned superset) ----------------------
-  const uint64_t vbeg = fstart + bm_bytes + uint64_t(G::W) * excl;
-  const uint64_t vend = vbeg + uint64_t(G::W) * tile_nnz;
-  const uint64_t abeg = vbeg & ~uint64_t(15), aend = a16(vend);
+  uint32_t woff = 0, nnz = 0;
+#pragma unroll
+  for (int w = 0; w < kWarps; w++) {
+    woff += w < warp ? s_woff[w] : 0;
+    nnz += s_woff[w];
+  }
+  const uint64_t vlast = vbeg + uint64_t(nnz) * G::W;
+  const uint64_t abeg = vbeg & ~uint64_t(15), aend = a16(vlast);
   const uint32_t d = uint32_t(vbeg - abeg);
-  const bool in_bounds = aend <= fstart + fbytes;
-  if (!in_bounds && tid == 0) set_error(err, kErrCorrupt);
+  const bool ok = aend <= fend && vbeg >= fstart && (vend == 0 || vend == vlast);
   if (tid == 0) {
-    const uint32_t bytes = in_bounds ? uint32_t(aend - abeg) : 0;
+    if (!ok) set_error(err, kErrCorrupt);
+    const uint32_t bytes = ok ? uint32_t(aend - abeg) : 0;
     if (bytes) {
       mbar_expect_tx(&s_bar, bytes);
       bulk_g2s(s_val, in + abeg, bytes, &s_bar);
     } else {
-      asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(
-                       static_cast<uint32_t>(__cvta_generic_to_shared(&s_bar)))
-                   : "memory");
+      mbar_arrive(&s_bar);
     }
   }
-  mbar_wait(&s_bar, 0);
-
-  // ---- 4. expand: each lane rebuilds EPV elements -> one 16-byte store --------------------
-  T* dst = outp + uint64_t(k) * F + tin;
-  uint32_t r = s_warp_off[warp];
+  mbar_wait(&s_bar, 1);
+  T* dst = outp + uint64_t(k) * F + uint64_t(j) * G::TILE;
+  uint32_t r = woff;
 #pragma unroll
   for (int q = 0; q < G::NCH; q++) {
     const uint32_t e0 = warp * G::PER_WARP + q * G::CHUNK + lane * G::EPV;
-    const uint32_t wbase = e0 / 32;  // first bitmap word of this chunk is (chunk start)/32
     const uint32_t cw0 = (warp * G::PER_WARP + q * G::CHUNK) / 32;
-    uint32_t before = 0, mine = 0;
+    const uint32_t myw = e0 / 32;
+    uint32_t before = 0, mine = 0, total = 0;
 #pragma unroll
-    for (int m = 0; m < G::EPV; m++) {  // the EPV words of this chunk
-      const uint32_t wd = s_bm[cw0 + m];
-      if (cw0 + m < wbase) before += __popc(wd);
-      if (cw0 + m == wbase) mine = wd;
+    for (int m = 0; m < G::EPV; m++) {
+      const uint32_t wi = cw0 + m;
+      uint32_t x = wi < nw ? s_bm[wi] : 0;
+      if (wi == nw - 1 && (tile_elems & 31)) x &= (1u << (tile_elems & 31)) - 1;
+      const uint32_t p = __popc(x);
+      before += wi < myw ? p : 0;
+      if (wi == myw) mine = x;
+      total += p;
     }
     const uint32_t sh = (lane % G::LPW) * G::EPV;
     const uint32_t b = (mine >> sh) & ((1u << G::EPV) - 1);
     uint32_t rank = r + before + __popc(mine & ((1u << sh) - 1));
     uint32_t w4[4] = {0, 0, 0, 0};
 #pragma unroll
-    for (int i = 0; i < G::EPV; i++) {
-      if (b & (1u << i)) {
+    for (int e = 0; e < G::EPV; e++) {
+      if ((b >> e) & 1) {
         uint32_t x;
         if constexpr (sizeof(T) == 4) x = *reinterpret_cast<const uint32_t*>(s_val + d + 4 * rank);
         else x = *reinterpret_cast<const uint16_t*>(s_val + d + 2 * rank);
-        if constexpr (sizeof(T) == 4) w4[i] = x;
-        else w4[i >> 1] |= x << ((i & 1) * 16);
+        if constexpr (sizeof(T) == 4) w4[e] = x;
+        else w4[e >> 1] |= x << ((e & 1) * 16);
         rank++;
       }
     }
-    uint32_t chunk_total = 0;
-#pragma unroll
-    for (int m = 0; m < G::EPV; m++) chunk_total += __popc(s_bm[cw0 + m]);
-    r += chunk_total;
-    if (!in_bounds) w4[0] = w4[1] = w4[2] = w4[3] = 0;
+    r += total;
+    if (!ok) w4[0] = w4[1] = w4[2] = w4[3] = 0;
     if (e0 + G::EPV <= tile_elems) {
       stg_stream(reinterpret_cast<uint4*>(dst + e0), make_uint4(w4[0], w4[1], w4[2], w4[3]));
     } else {
-      for (int i = 0; i < G::EPV; i++)
-        if (e0 + i < tile_elems) {
-          if constexpr (sizeof(T) == 4) dst[e0 + i] = w4[i];
-          else dst[e0 + i] = T((w4[i >> 1] >> ((i & 1) * 16)) & 0xFFFFu);
+      for (int e = 0; e < G::EPV; e++)
+        if (e0 + e < tile_elems) {
+          if constexpr (sizeof(T) == 4) dst[e0 + e] = w4[e];
+          else dst[e0 + e] = T((w4[e >> 1] >> ((e & 1) * 16)) & 0xFFFFu);
         }
     }
   }
 }
 
 // ------------------------------------------------------------------------------------------
-template <typename T>
-static cudaError_t launch_zvc_compress_t(const void* in, uint64_t n, uint64_t F, uint8_t* out, uint64_t* out_size,
-                                         const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st) {
-  using G = ZvcGeom<T>;
-  const uint32_t K = uint32_t(cdiv(n, F));
-  const uint32_t tpf = uint32_t(cdiv(F, G::TILE));
-  const uint32_t tiles = (K - 1) * tpf + uint32_t(cdiv(frame_len(n, F, K - 1), G::TILE));
-  const int smem = kTileBytes + 16;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(zvc_compress_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    attr = true;
-  }
-  zvc_compress_kernel<T><<<tiles, kThreads, smem, st>>>(static_cast<const T*>(in), n, F, K, tpf, tiles, out,
-                                                        out_size, sc, epoch, dtype);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
-                                const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st) {
-  return w == 4 ? launch_zvc_compress_t<uint32_t>(in, n, F, out, out_size, sc, epoch, dtype, st)
-                : launch_zvc_compress_t<uint16_t>(in, n, F, out, out_size, sc, epoch, dtype, st);
-}
-
 uint32_t zvc_tiles(uint64_t n, int w, uint64_t F, uint32_t k0, uint32_t k1, uint32_t* tpf_out) {
   const uint32_t TILE = kTileBytes / w;
   const uint32_t tpf = uint32_t(cdiv(F, TILE));
@@ -401,29 +660,105 @@ uint32_t zvc_tiles(uint64_t n, int w, uint64_t F, uint32_t k0, uint32_t k1, uint
   return (k1 - 1 - k0) * tpf + uint32_t(cdiv(frame_len(n, F, k1 - 1), TILE));
 }
 
+static int prof_enabled() {
+  static int p = -1;
+  if (p < 0) p = getenv("CSWAP_ZVC_PROF") ? 1 : 0;
+  return p;
+}
+
+static int sm_count() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  return sms;
+}
+
+template <typename T, int S>
+static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uint8_t* out, uint64_t* out_size,
+                                     const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st) {
+  using L = CompressSmem<T, S>;
+  const uint32_t K = uint32_t(cdiv(n, F));
+  uint32_t tpf;
+  const uint32_t tiles = zvc_tiles(n, sizeof(T), F, 0, K, &tpf);
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(zvc_compress_persistent<T, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, L::bytes);
+    attr = true;
+  }
+  const uint32_t per_sm = L::ctas_per_sm;
+  // per-frame and per-group (tiles, nnz) accumulators
+  cudaMemsetAsync(sc.aux2, 0, (uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32)) * 8, st);
+  const uint32_t grid = std::min<uint32_t>(tiles, uint32_t(sm_count()) * per_sm);
+  zvc_compress_persistent<T, S><<<grid, compress_threads<S>(), L::bytes, st>>>(
+      static_cast<const T*>(in), n, F, K, tpf, tiles, out, out_size, sc, epoch, dtype, prof_enabled());
+  if (prof_enabled()) {
+    unsigned long long h[16];
+    cudaStreamSynchronize(st);
+    cudaMemcpyFromSymbol(h, g_zprof, sizeof(h));
+    fprintf(stderr,
+            "[zprof] grid=%u tiles=%u | per-tile cycles: producer_wait_empty=%.0f counter_wait_full=%.0f "
+            "resolver_wait_cnt=%.0f resolver_lookback=%.0f | consumer(tid0): wait_off=%.0f finish=%.0f "
+            "wait_full=%.0f prep=%.0f\n",
+            grid, tiles, h[0] / double(tiles), h[1] / double(tiles), h[2] / double(tiles), h[3] / double(tiles),
+            h[5] / double(tiles), h[6] / double(tiles), h[7] / double(tiles), h[8] / double(tiles));
+    memset(h, 0, sizeof(h));
+    cudaMemcpyToSymbol(g_zprof, h, sizeof(h));
+  }
+  return cudaGetLastError();
+}
+
+static int stages_cfg() {
+  static int s = -1;
+  if (s < 0) {
+    const char* e = getenv("CSWAP_ZVC_STAGES");
+    s = e ? atoi(e) : 3;
+    if (s < 2 || s > 6) s = 3;
+  }
+  return s;
+}
+
+template <typename T>
+static cudaError_t launch_compress_t(const void* in, uint64_t n, uint64_t F, uint8_t* out, uint64_t* out_size,
+                                     const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st) {
+  switch (stages_cfg()) {
+    case 2: return launch_compress_s<T, 2>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    case 4: return launch_compress_s<T, 4>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    case 5: return launch_compress_s<T, 5>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    default: return launch_compress_s<T, 3>(in, n, F, out, out_size, sc, epoch, dtype, st);
+  }
+}
+
+cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
+                                const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st) {
+  return w == 4 ? launch_compress_t<uint32_t>(in, n, F, out, out_size, sc, epoch, dtype, st)
+                : launch_compress_t<uint16_t>(in, n, F, out, out_size, sc, epoch, dtype, st);
+}
+
 template <typename T>
 static cudaError_t launch_zvc_decompress_t(const uint8_t* in, void* out, uint64_t n, uint64_t F, uint32_t k0,
-                                           uint32_t k1, const Scratch& sc, uint32_t epoch, uint32_t* err,
-                                           cudaStream_t st) {
-  const uint32_t K = uint32_t(cdiv(n, F));
+                                           uint32_t k1, const Scratch& sc, uint32_t* err, cudaStream_t st) {
   uint32_t tpf;
   const uint32_t tiles = zvc_tiles(n, sizeof(T), F, k0, k1, &tpf);
   if (!tiles) return cudaSuccess;
+  zvc_count_kernel<T><<<(tiles + kWarps - 1) / kWarps, kThreads, 0, st>>>(in, n, F, tpf, k0, tiles, sc, err);
+  zvc_scan_kernel<T><<<k1 - k0, 1024, 0, st>>>(n, F, tpf, k0, sc, err);
   const int smem = kTileBytes + 32;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(zvc_decompress_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(zvc_expand_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
-  zvc_decompress_kernel<T><<<tiles, kThreads, smem, st>>>(in, static_cast<T*>(out), n, F, K, tpf, k0, tiles, sc,
-                                                          epoch, err);
+  zvc_expand_kernel<T><<<tiles, kThreads, smem, st>>>(in, static_cast<T*>(out), n, F, tpf, k0, sc, err);
   return cudaGetLastError();
 }
 
 cudaError_t launch_zvc_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
-                                  uint32_t k1, const Scratch& sc, uint32_t epoch, uint32_t* err, cudaStream_t st) {
-  return w == 4 ? launch_zvc_decompress_t<uint32_t>(in, out, n, F, k0, k1, sc, epoch, err, st)
-                : launch_zvc_decompress_t<uint16_t>(in, out, n, F, k0, k1, sc, epoch, err, st);
+                                  uint32_t k1, const Scratch& sc, uint32_t /*epoch*/, uint32_t* err, cudaStream_t st) {
+  return w == 4 ? launch_zvc_decompress_t<uint32_t>(in, out, n, F, k0, k1, sc, err, st)
+                : launch_zvc_decompress_t<uint16_t>(in, out, n, F, k0, k1, sc, err, st);
 }
 
 }  // namespace cswap

@@ -67,6 +67,11 @@ class Decision(ctypes.Structure):
                 "t_dc": list(self.t_dc)}
 
 
+class KernelRecord(ctypes.Structure):
+    _fields_ = [("codec", ctypes.c_int32), ("direction", ctypes.c_int32), ("raw_bytes", ctypes.c_uint64),
+                ("comp_bytes", ctypes.c_uint64), ("ms", ctypes.c_double)]
+
+
 _vp, _u64, _u32, _i, _d = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int, ctypes.c_double
 _P = ctypes.POINTER
 _SIGS = {
@@ -91,6 +96,9 @@ _SIGS = {
     "cswap_handle_free": (None, [_vp]),
     "cswap_fit_time_model": (_i, [_P(_d), _P(_d), _P(_d), _u64, _P(_d)]),
     "cswap_fit_link": (_i, [_P(_d), _P(_d), _u64, _P(_d), _P(_d)]),
+    "cswap_fit_linear": (_i, [_P(_d), _P(_d), _u64, _u32, _P(_d)]),
+    "cswap_set_kernel_timing": (_i, [_i]),
+    "cswap_collect_kernel_timing": (_u64, [_P(KernelRecord), _u64]),
     "cswap_status_string": (ctypes.c_char_p, [_i]),
     "cswap_last_error": (ctypes.c_char_p, []),
     "cswap_kernel_launches": (_u64, []),
@@ -274,6 +282,26 @@ def fit_link(nbytes, t):
     a, bw = ctypes.c_double(), ctypes.c_double()
     _check(_L.cswap_fit_link(A(*nbytes), A(*t), m, ctypes.byref(a), ctypes.byref(bw)), "cswap_fit_link")
     return a.value, bw.value
+
+
+def fit_linear(X, y):
+    """OLS y = X beta; X is a list of rows (p <= 8 columns)."""
+    m, p = len(X), len(X[0])
+    flat = (ctypes.c_double * (m * p))(*[v for row in X for v in row])
+    beta = (ctypes.c_double * p)()
+    _check(_L.cswap_fit_linear(flat, (ctypes.c_double * m)(*y), m, p, beta), "cswap_fit_linear")
+    return list(beta)
+
+
+def set_kernel_timing(enable: bool):
+    _check(_L.cswap_set_kernel_timing(1 if enable else 0), "cswap_set_kernel_timing")
+
+
+def collect_kernel_timing(cap: int = 1 << 16):
+    buf = (KernelRecord * cap)()
+    k = int(_L.cswap_collect_kernel_timing(buf, cap))
+    return [{"codec": r.codec, "direction": r.direction, "raw_bytes": r.raw_bytes, "comp_bytes": r.comp_bytes,
+             "ms": r.ms} for r in buf[:k]]
 
 
 def kernel_launches() -> int:
