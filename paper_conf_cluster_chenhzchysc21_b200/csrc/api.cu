@@ -226,6 +226,8 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
     cudaFree(b.sc.aux2);
     cudaFree(b.sc.err);
     cudaFree(b.sc.tbuf);
+    cudaFree(b.sc.tbuf2);
+    cudaFree(b.sc.aux3);
   }
   tiles = std::max(tiles, b.sc.cap_tiles * 2);
   aux = std::max(aux, b.sc.cap_aux * 2);
@@ -235,6 +237,8 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
   CU(cudaMalloc(&b.sc.aux2, aux * 8));
   CU(cudaMalloc(&b.sc.err, 64));
   CU(cudaMalloc(&b.sc.tbuf, tiles * 8));
+  CU(cudaMalloc(&b.sc.tbuf2, tiles * 8));
+  CU(cudaMalloc(&b.sc.aux3, aux * 8));
   CU(cudaMemset(b.sc.status, 0, tiles * 8));
   CU(cudaMemset(b.sc.tickets, 0, kEpochs * 4));
   CU(cudaMemset(b.sc.err, 0, 64));
@@ -362,16 +366,15 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       return cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, L.b->sc, L.epoch(), dtype, st), "zvc_compress");
     }
     case CSWAP_CODEC_RLE: {
-      Lease L(*c, st, rle_tiles(n, w, F) + 2, std::max<uint64_t>(K, rle_tiles(n, w, F)) + 2);
+      Lease L(*c, st, rle_tiles(n, w, F) + 2, uint64_t(K) + 2);
       TRY(L.status);
-      c->launches += 3;
+      c->launches += 4;
       return cuda_status(launch_rle_compress(in, n, w, F, out, out_size, L.b->sc, L.epoch(), dtype, st), "rle_compress");
     }
     case CSWAP_CODEC_CSR: {
-      const uint64_t rows = (n + f.csr_row - 1) / f.csr_row + K;
-      Lease L(*c, st, 1024, std::max<uint64_t>(rows, K) + 2);
+      Lease L(*c, st, rle_tiles(n, w, F) + 2, uint64_t(K) + 2);
       TRY(L.status);
-      c->launches += 3;
+      c->launches += 4;
       return cuda_status(launch_csr_compress(in, n, w, F, f.csr_row, out, out_size, L.b->sc, L.epoch(), dtype, st),
                          "csr_compress");
     }
@@ -523,6 +526,8 @@ cswap_status cswap_shutdown(void) {
     cudaFree(b.sc.aux2);
     cudaFree(b.sc.err);
     cudaFree(b.sc.tbuf);
+    cudaFree(b.sc.tbuf2);
+    cudaFree(b.sc.aux3);
     cudaEventDestroy(b.ev);
   }
   cudaFree(c->dev_err);

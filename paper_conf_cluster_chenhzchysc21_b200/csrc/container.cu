@@ -46,6 +46,58 @@ cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, 
   return cudaGetLastError();
 }
 
+// ---- frame table finalize (multi-pass codecs): frame_bytes[k] in fbytes[k] -> frame table,
+// frame starts (fstart[k]), header, padding, *out_size.  One CTA.
+__global__ void __launch_bounds__(1024) finalize_kernel(uint8_t* out, int codec, int dtype, uint64_t n, uint64_t F,
+                                                        uint32_t param, const uint64_t* fbytes, uint64_t* fstart,
+                                                        uint64_t* out_size) {
+  __shared__ uint64_t s_w[33];
+  const uint32_t K = uint32_t(cdiv(n, F));
+  const uint64_t base = data_start(K);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t carry = 0;
+  for (uint32_t c = 0; c < K; c += blockDim.x) {
+    const uint32_t k = c + threadIdx.x;
+    const uint64_t fb = k < K ? fbytes[k] : 0;
+    uint64_t inc = fb;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += y;
+    }
+    if (lane == 31) s_w[warp] = inc;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint64_t acc = 0;
+      for (int w = 0; w < int(blockDim.x / 32); w++) {
+        const uint64_t x = s_w[w];
+        s_w[w] = acc;
+        acc += x;
+      }
+      s_w[32] = acc;
+    }
+    __syncthreads();
+    if (k < K) {
+      fstart[k] = base + carry + s_w[warp] + inc - fb;
+      reinterpret_cast<uint64_t*>(out + 64)[k] = fb;
+    }
+    carry += s_w[32];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    const uint64_t total = base + carry;
+    write_header(out, codec, dtype, n, F, K, param, total);
+    for (uint64_t b = 64 + 8ull * K; b < base; b += 8) *reinterpret_cast<uint64_t*>(out + b) = 0;
+    *out_size = total;
+  }
+}
+
+cudaError_t launch_finalize(uint8_t* out, int codec, int dtype, uint64_t n, uint64_t F, uint32_t param,
+                            const Scratch& sc, uint64_t* out_size, cudaStream_t st) {
+  finalize_kernel<<<1, 1024, 0, st>>>(out, codec, dtype, n, F, param, sc.aux2, sc.aux, out_size);
+  return cudaGetLastError();
+}
+
 // ---- error word merge (device scratch word -> caller's word, first error wins) ---------------
 __global__ void err_merge_kernel(const uint32_t* src, uint32_t* dst) {
   const uint32_t v = *src;

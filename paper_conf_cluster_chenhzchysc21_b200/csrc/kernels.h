@@ -12,6 +12,9 @@ cudaError_t launch_header_only(uint8_t* out, int codec, int dtype, uint64_t F, u
                                cudaStream_t st);
 cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
                         uint32_t param, const Scratch& sc, uint32_t* err, cudaStream_t st);
+// frame_bytes in sc.aux2[k] -> frame table, frame starts in sc.aux[k], header, *out_size
+cudaError_t launch_finalize(uint8_t* out, int codec, int dtype, uint64_t n, uint64_t F, uint32_t param,
+                            const Scratch& sc, uint64_t* out_size, cudaStream_t st);
 cudaError_t launch_err_merge(const uint32_t* src, uint32_t* dst, cudaStream_t st);
 cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, int dtype, uint8_t* out,
                                  uint64_t* out_size, cudaStream_t st);
