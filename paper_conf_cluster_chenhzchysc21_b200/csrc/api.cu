@@ -382,11 +382,10 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       const uint64_t blocks = lz4_scratch_bytes(n, w, F, f.lz4_block);
       uint8_t* slots = nullptr;
       CU(cudaMallocAsync(&slots, blocks, st));
-      uint64_t nblk = 0;
-      for (uint32_t k = 0; k < K; k++) nblk += (std::min<uint64_t>(F, n - uint64_t(k) * F) * w + f.lz4_block - 1) / f.lz4_block;
+      const uint64_t bidx = uint64_t(K) * ((F * w + f.lz4_block - 1) / f.lz4_block);  // block index k*bpf + b
       cswap_status s;
       {
-        Lease L(*c, st, 1024, nblk + K + 2);
+        Lease L(*c, st, bidx + 2, uint64_t(K) + 2);
         TRY(L.status);
         c->launches += 3;
         s = cuda_status(launch_lz4_compress(in, n, w, F, f.lz4_block, out, out_size, slots, L.b->sc, dtype, st),
@@ -427,6 +426,7 @@ uint64_t decompress_tiles(uint64_t n, int w, const cswap_format& f) {
   const uint64_t F = f.frame_elems, K = (n + F - 1) / F;
   uint64_t t = zvc_tiles(n, w, F, 0, uint32_t(K), nullptr);
   t = std::max<uint64_t>(t, rle_tiles(n, w, F) + 2);
+  t = std::max<uint64_t>(t, K * ((F * w + f.lz4_block - 1) / f.lz4_block));  // LZ4 block index k*bpf + b
   return t + 2;
 }
 uint64_t decompress_aux(uint64_t n, int w, const cswap_format& f) {

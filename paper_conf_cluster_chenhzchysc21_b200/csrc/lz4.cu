@@ -1,0 +1,340 @@
+// lz4.cu — LZ4 block codec for sm_100a.
+//
+// PAPER.md:220-222 (§IV-E): "LZ4 uses a dictionary-matching stage to reduce data size. For
+// example, a string (abcde_bcde) can be compressed as (abcde_(5,4)), where 5 denotes the position
+// how far back the redundant string (bcde) can be found and 4 denotes the length of matched
+// string."  [25] = nvcomp: independent blocks.  Reading R6 / DESIGN.md §3.2: every
+// B-byte block is an LZ4 *block-format* stream produced by the canonical greedy parse
+// (MINMATCH 4, MFLIMIT 12, LASTLITERALS 5, HASHLOG 12, lookup-then-insert at every scanned
+// position, nothing inserted inside matches).  Frame: u32 csize[nblk] pad16 | blocks | pad16.
+//
+// Compress: one warp per block, block + 4096-entry u16 hash table in shared memory.  The warp
+// scans 32 consecutive positions at a time: lane j's candidate is the latest earlier lane with the
+// same hash (__match_any_sync) else the table entry; the first lane whose candidate verifies ends
+// the batch; lanes up to it insert (latest lane per hash wins).  This is exactly the sequential
+// parse.  Matches are extended 32 bytes per step; sequences are written by the
+// whole warp into a per-block scratch slot.  Then: per-frame scan of block sizes -> frame table
+// -> pack (one CTA per block).
+// Decompress: per-frame scan of csize -> block offsets; one warp per block decodes into shared
+// memory (literal and match copies 32 bytes per step, short-offset matches by pattern
+// replication) with every read and write bounds-checked, then stores the block with 16-byte stores.
+#include "kernels.h"
+#include "tile_common.cuh"
+
+namespace cswap {
+
+constexpr uint32_t kLz4MaxBlock = 65536;
+constexpr uint32_t kLz4SlotBytes = 65824;  // >= L + L/255 + 16 for L = 65536, multiple of 16
+constexpr uint16_t kLz4Empty = 0xFFFF;     // positions <= L-12 < 0xFFFF are the only ones inserted
+
+__device__ __forceinline__ uint32_t le32_smem(const uint8_t* s, uint32_t p) {  // s 4-aligned, +8 pad
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(s);
+  const uint32_t a = w[p >> 2], b = w[(p >> 2) + 1];
+  return __funnelshift_r(a, b, (p & 3) * 8);
+}
+
+// Writes `len` bytes of `val` at out[op..] with the whole warp.
+__device__ __forceinline__ void warp_fill(uint8_t* out, uint32_t op, uint32_t len, uint8_t val, int lane) {
+  for (uint32_t q = lane; q < len; q += 32) out[op + q] = val;
+}
+
+// LZ4 length continuation for v >= 0 (the part beyond the token nibble): bytes of 255 + remainder
+__device__ __forceinline__ uint32_t put_len_ext(uint8_t* out, uint32_t op, uint32_t v, int lane) {
+  const uint32_t n255 = v / 255;
+  warp_fill(out, op, n255, 255, lane);
+  if (lane == 0) out[op + n255] = uint8_t(v - 255 * n255);
+  return op + n255 + 1;
+}
+
+// Emit one sequence (literals src[anchor, anchor+nlit), optional match) at out[op]; returns new op.
+__device__ __forceinline__ uint32_t emit_seq(uint8_t* out, uint32_t op, const uint8_t* src, uint32_t anchor,
+                                             uint32_t nlit, bool has_match, uint32_t offset, uint32_t mlen, int lane) {
+  const uint32_t tl = nlit < 15 ? nlit : 15;
+  const uint32_t tm = has_match ? ((mlen - 4) < 15 ? (mlen - 4) : 15) : 0;
+  if (lane == 0) out[op] = uint8_t((tl << 4) | tm);
+  op++;
+  if (nlit >= 15) op = put_len_ext(out, op, nlit - 15, lane);
+  for (uint32_t q = lane; q < nlit; q += 32) out[op + q] = src[anchor + q];
+  op += nlit;
+  if (has_match) {
+    if (lane == 0) {
+      out[op] = uint8_t(offset & 0xFF);
+      out[op + 1] = uint8_t(offset >> 8);
+    }
+    op += 2;
+    if (mlen - 4 >= 15) op = put_len_ext(out, op, mlen - 4 - 15, lane);
+  }
+  return op;
+}
+
+// one warp per block; blocks indexed globally (frame-major), block b of frame k covers bytes
+// [b*B, min((b+1)*B, Fk*w)) of the frame
+__global__ void __launch_bounds__(32) lz4_compress_kernel(const uint8_t* __restrict__ in, uint64_t n, int w,
+                                                          uint64_t F, uint32_t B, uint32_t bpf, uint8_t* slots,
+                                                          uint64_t* csize) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  uint8_t* s_src = smem;                                              // B + 16 bytes
+  uint16_t* s_tab = reinterpret_cast<uint16_t*>(smem + kLz4MaxBlock + 16);  // 4096 entries
+  const int lane = threadIdx.x;
+  const uint32_t blk = blockIdx.x;
+  const uint32_t k = blk / bpf, b = blk % bpf;
+  const uint64_t fbytes = frame_len(n, F, k) * uint64_t(w);
+  const uint32_t L = uint32_t(umin64(B, fbytes - uint64_t(b) * B));
+  const uint8_t* src = in + uint64_t(k) * F * w + uint64_t(b) * B;
+  // stage the block (16-byte vectors; B and every block start are 16-aligned, the tail is scalar)
+  const uint32_t nv = L / 16;
+  for (uint32_t v = lane; v < nv; v += 32)
+    reinterpret_cast<uint4*>(s_src)[v] = ldg_stream(reinterpret_cast<const uint4*>(src) + v);
+  for (uint32_t q = nv * 16 + lane; q < L + 16; q += 32) s_src[q] = q < L ? src[q] : 0;
+  for (uint32_t h = lane; h < 4096; h += 32) s_tab[h] = kLz4Empty;
+  __syncwarp();
+  uint8_t* out = slots + uint64_t(blk) * kLz4SlotBytes;
+  const uint32_t lt = (1u << lane) - 1u;
+  uint32_t anchor = 0, i = 0, op = 0;
+  if (L >= 13) {
+    const uint32_t limit = L - 12;  // last position that may start a match
+    while (i <= limit) {
+      const uint32_t pos = i + lane;
+      const bool active = pos <= limit;
+      const uint32_t v = active ? le32_smem(s_src, pos) : 0;
+      const uint32_t h = active ? (v * 2654435761u) >> 20 : 0x10000u + lane;
+      const uint32_t same = __match_any_sync(0xffffffffu, h);
+      const uint32_t earlier = same & lt;
+      uint32_t cand = kLz4Empty;
+      if (active) cand = earlier ? i + (31 - __clz(earlier)) : s_tab[h];
+      const bool ok = active && cand != kLz4Empty && le32_smem(s_src, cand) == v;
+      const uint32_t mm = __ballot_sync(0xffffffffu, ok);
+      // lanes that insert: up to the first matching lane (all active lanes if none matched);
+      // within a hash group the latest inserting lane wins
+      const int f = mm ? __ffs(mm) - 1 : 31;
+      const uint32_t upto = f == 31 ? 0xffffffffu : ((2u << f) - 1u);
+      const uint32_t later = same & ~lt & ~(1u << lane) & upto;
+      __syncwarp();
+      if (active && (upto >> lane & 1u) && later == 0) s_tab[h] = uint16_t(pos);
+      __syncwarp();
+      if (!mm) {
+        i += 32;
+        continue;
+      }
+      const uint32_t mpos = i + f;
+      const uint32_t c = __shfl_sync(0xffffffffu, cand, f);
+      uint32_t len = 4;
+      while (true) {  // extend while mpos+len < L-5 and bytes agree, 32 bytes per step
+        const uint32_t q = mpos + len + lane;
+        const bool eq = q < L - 5 && s_src[c + len + lane] == s_src[q];
+        const uint32_t ne = __ballot_sync(0xffffffffu, !eq);
+        if (ne) {
+          len += __ffs(ne) - 1;
+          break;
+        }
+        len += 32;
+      }
+      op = emit_seq(out, op, s_src, anchor, mpos - anchor, true, mpos - c, len, lane);
+      i = mpos + len;
+      anchor = i;
+    }
+  }
+  op = emit_seq(out, op, s_src, anchor, L - anchor, false, 0, 0, lane);
+  if (lane == 0) csize[blk] = op;
+}
+
+// one CTA per frame: block offsets inside the frame's block section (tbuf), frame_bytes (aux2)
+__global__ void __launch_bounds__(1024) lz4_scan_kernel(uint64_t n, int w, uint64_t F, uint32_t B, uint32_t bpf,
+                                                        Scratch sc) {
+  __shared__ uint64_t s_tmp[33];
+  const uint32_t k = blockIdx.x;
+  const uint32_t nb = uint32_t(cdiv(frame_len(n, F, k) * uint64_t(w), B));
+  uint64_t* cs = sc.tbuf + uint64_t(k) * bpf;
+  uint64_t* off = sc.tbuf2 + uint64_t(k) * bpf;
+  uint64_t carry = 0;
+  for (uint32_t c0 = 0; c0 < nb; c0 += blockDim.x) {
+    const uint32_t j = c0 + threadIdx.x;
+    const uint64_t v = j < nb ? cs[j] : 0;
+    uint64_t tot;
+    const uint64_t ex = block_excl_sum_u64(v, s_tmp, &tot);
+    if (j < nb) off[j] = carry + ex;
+    carry += tot;
+  }
+  if (threadIdx.x == 0) sc.aux2[k] = a16(4ull * nb) + a16(carry);
+}
+
+// one CTA per block: copy the slot to its place, write csize[b], pads
+__global__ void __launch_bounds__(256) lz4_pack_kernel(uint64_t n, int w, uint64_t F, uint32_t B, uint32_t bpf,
+                                                       const uint8_t* slots, uint8_t* out, Scratch sc) {
+  const uint32_t blk = blockIdx.x;
+  const uint32_t k = blk / bpf, b = blk % bpf;
+  const uint32_t nb = uint32_t(cdiv(frame_len(n, F, k) * uint64_t(w), B));
+  const uint64_t fstart = sc.aux[k];
+  const uint64_t cs = sc.tbuf[blk];
+  uint8_t* dst = out + fstart + a16(4ull * nb) + sc.tbuf2[blk];
+  const uint8_t* src = slots + uint64_t(blk) * kLz4SlotBytes;
+  for (uint32_t q = threadIdx.x; q < cs; q += blockDim.x) dst[q] = src[q];
+  if (threadIdx.x == 0) reinterpret_cast<uint32_t*>(out + fstart)[b] = uint32_t(cs);
+  if (threadIdx.x == 1 && b == nb - 1) {  // pads of the csize section and of the block section
+    for (uint64_t q = 4ull * nb; q < a16(4ull * nb); q++) out[fstart + q] = 0;
+    const uint64_t end = a16(4ull * nb) + sc.tbuf2[blk] + cs;
+    for (uint64_t q = end; q < a16(end); q++) out[fstart + q] = 0;
+  }
+}
+
+uint64_t lz4_scratch_bytes(uint64_t n, int w, uint64_t F, uint32_t B) {
+  const uint64_t K = cdiv(n, F);
+  uint64_t nblk = 0;
+  for (uint64_t k = 0; k < K; k++) nblk += cdiv(frame_len(n, F, k) * w, B);
+  return (nblk + 1) * kLz4SlotBytes;
+}
+
+static uint32_t lz4_blocks(uint64_t n, int w, uint64_t F, uint32_t B, uint32_t* bpf_out) {
+  const uint32_t K = uint32_t(cdiv(n, F));
+  const uint32_t bpf = uint32_t(cdiv(F * w, B));
+  if (bpf_out) *bpf_out = bpf;
+  return (K - 1) * bpf + uint32_t(cdiv(frame_len(n, F, K - 1) * w, B));
+}
+
+cudaError_t launch_lz4_compress(const void* in, uint64_t n, int w, uint64_t F, uint32_t B, uint8_t* out,
+                                uint64_t* out_size, uint8_t* slots, const Scratch& sc, int dtype, cudaStream_t st) {
+  const uint32_t K = uint32_t(cdiv(n, F));
+  uint32_t bpf;
+  const uint32_t nblk = lz4_blocks(n, w, F, B, &bpf);
+  const int smem = kLz4MaxBlock + 16 + 4096 * 2;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(lz4_compress_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    attr = true;
+  }
+  lz4_compress_kernel<<<nblk, 32, smem, st>>>(static_cast<const uint8_t*>(in), n, w, F, B, bpf, slots, sc.tbuf);
+  lz4_scan_kernel<<<K, 1024, 0, st>>>(n, w, F, B, bpf, sc);
+  cudaError_t e = launch_finalize(out, kLZ4, dtype, n, F, B, sc, out_size, st);
+  if (e != cudaSuccess) return e;
+  lz4_pack_kernel<<<nblk, 256, 0, st>>>(n, w, F, B, bpf, slots, out, sc);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------------------------------
+// decompress
+// ------------------------------------------------------------------------------------------
+// one CTA per frame: validate csize against frame_bytes, block offsets -> tbuf2
+__global__ void __launch_bounds__(1024) lz4_dscan_kernel(const uint8_t* __restrict__ in, uint64_t n, int w,
+                                                         uint64_t F, uint32_t B, uint32_t bpf, uint32_t k0, Scratch sc,
+                                                         uint32_t* err) {
+  __shared__ uint64_t s_tmp[33];
+  if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
+  const uint32_t k = k0 + blockIdx.x;
+  const uint32_t nb = uint32_t(cdiv(frame_len(n, F, k) * uint64_t(w), B));
+  const uint64_t fstart = sc.aux[k], fb = sc.aux2[k];
+  if (a16(4ull * nb) > fb) {
+    if (threadIdx.x == 0) set_error(err, kErrCorrupt);
+    return;
+  }
+  const uint32_t* cs = reinterpret_cast<const uint32_t*>(in + fstart);
+  uint64_t* off = sc.tbuf2 + uint64_t(k) * bpf;
+  uint64_t* csz = sc.tbuf + uint64_t(k) * bpf;
+  uint64_t carry = 0;
+  for (uint32_t c0 = 0; c0 < nb; c0 += blockDim.x) {
+    const uint32_t j = c0 + threadIdx.x;
+    const uint64_t v = j < nb ? cs[j] : 0;
+    uint64_t tot;
+    const uint64_t ex = block_excl_sum_u64(v, s_tmp, &tot);
+    if (j < nb) {
+      off[j] = carry + ex;
+      csz[j] = v;
+    }
+    carry += tot;
+  }
+  if (threadIdx.x == 0 && a16(4ull * nb) + a16(carry) != fb) set_error(err, kErrCorrupt);
+}
+
+__global__ void __launch_bounds__(32) lz4_decode_kernel(const uint8_t* __restrict__ in, uint8_t* __restrict__ outp,
+                                                        uint64_t n, int w, uint64_t F, uint32_t B, uint32_t bpf,
+                                                        uint32_t k0, Scratch sc, uint32_t* err) {
+  extern __shared__ __align__(16) uint8_t s_out[];  // B bytes
+  if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
+  const int lane = threadIdx.x;
+  const uint32_t k = k0 + blockIdx.x / bpf, b = blockIdx.x % bpf;
+  const uint64_t fbytes = frame_len(n, F, k) * uint64_t(w);
+  const uint32_t nb = uint32_t(cdiv(fbytes, B));
+  if (b >= nb) return;
+  const uint32_t L = uint32_t(umin64(B, fbytes - uint64_t(b) * B));
+  const uint64_t blk = uint64_t(k) * bpf + b;
+  const uint64_t fstart = sc.aux[k], fb = sc.aux2[k];
+  const uint64_t cs = sc.tbuf[blk];
+  const uint64_t start = a16(4ull * nb) + sc.tbuf2[blk];
+  bool bad = start + cs > fb;
+  const uint8_t* ip0 = in + fstart + start;
+  uint64_t ip = 0;
+  uint32_t op = 0;
+  auto rd = [&](uint64_t at) -> uint32_t { return at < cs ? ip0[at] : 0u; };
+  while (!bad) {
+    if (ip >= cs) { bad = true; break; }
+    const uint32_t token = rd(ip++);
+    uint32_t nlit = token >> 4;
+    if (nlit == 15) {
+      uint32_t x;
+      do {
+        if (ip >= cs) { bad = true; break; }
+        x = rd(ip++);
+        nlit += x;
+      } while (x == 255);
+      if (bad) break;
+    }
+    if (ip + nlit > cs || op + nlit > L) { bad = true; break; }
+    for (uint32_t q = lane; q < nlit; q += 32) s_out[op + q] = ip0[ip + q];
+    ip += nlit;
+    op += nlit;
+    __syncwarp();
+    if (ip == cs) break;  // last sequence: literals only
+    if (ip + 2 > cs) { bad = true; break; }
+    const uint32_t offset = rd(ip) | (rd(ip + 1) << 8);
+    ip += 2;
+    uint32_t mlen = token & 15;
+    if (mlen == 15) {
+      uint32_t x;
+      do {
+        if (ip >= cs) { bad = true; break; }
+        x = rd(ip++);
+        mlen += x;
+      } while (x == 255);
+      if (bad) break;
+    }
+    mlen += 4;
+    if (offset == 0 || offset > op || op + mlen > L) { bad = true; break; }
+    if (offset >= 32) {  // non-overlapping within a 32-byte step
+      for (uint32_t q = 0; q < mlen; q += 32) {
+        if (q + lane < mlen) s_out[op + q + lane] = s_out[op + q + lane - offset];
+        __syncwarp();
+      }
+    } else {  // short offset: the match repeats the last `offset` bytes
+      const uint32_t base = op - offset;
+      for (uint32_t q = lane; q < mlen; q += 32) s_out[op + q] = s_out[base + (q % offset)];
+    }
+    op += mlen;
+    __syncwarp();
+  }
+  if (!bad && op != L) bad = true;
+  if (__any_sync(0xffffffffu, bad)) {
+    if (lane == 0) set_error(err, kErrCorrupt);
+    return;
+  }
+  __syncwarp();
+  uint8_t* dst = outp + uint64_t(k) * F * w + uint64_t(b) * B;
+  const uint32_t nv = L / 16;
+  for (uint32_t v = lane; v < nv; v += 32) stg_stream(reinterpret_cast<uint4*>(dst) + v, reinterpret_cast<const uint4*>(s_out)[v]);
+  for (uint32_t q = nv * 16 + lane; q < L; q += 32) dst[q] = s_out[q];
+}
+
+cudaError_t launch_lz4_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t B,
+                                  uint32_t k0, uint32_t k1, const Scratch& sc, uint32_t* err, cudaStream_t st) {
+  if (k1 <= k0) return cudaSuccess;
+  const uint32_t bpf = uint32_t(cdiv(F * w, B));
+  lz4_dscan_kernel<<<k1 - k0, 1024, 0, st>>>(in, n, w, F, B, bpf, k0, sc, err);
+  const int smem = kLz4MaxBlock;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(lz4_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    attr = true;
+  }
+  lz4_decode_kernel<<<(k1 - k0) * bpf, 32, B, st>>>(in, static_cast<uint8_t*>(out), n, w, F, B, bpf, k0, sc, err);
+  return cudaGetLastError();
+}
+
+}  // namespace cswap

@@ -2,7 +2,7 @@
 product C ABI.  No method arithmetic here."""
 import numpy as np
 
-IMPLEMENTED = (0, 1, 2, 3)  # codecs with CUDA kernels in this build (NONE, ZVC, RLE, CSR)
+IMPLEMENTED = (0, 1, 2, 3, 4)  # codecs with CUDA kernels in this build (all)
 
 
 def lib():
