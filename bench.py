@@ -26,7 +26,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "compressed swap-out+in latency & codec GB/s vs HBM roofline, 1/2/4/8 B200"
 CALIB_PATH = os.path.join(ROOT, "calib", "b200.json")
-NCU_SUMMARY = os.path.join(ROOT, "profiles", "ncu_zvc_r01.json")
+NCU_SUMMARY = os.path.join(ROOT, "profiles", "ncu_r01.json")
 
 
 def log(*a):
@@ -115,7 +115,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
     tensors, outs, sizes = [], [], []
     for i, (name, shape, s) in enumerate(tensors_spec):
         n = synth.numel(shape)
-        tensors.append(synth.relu_iid_torch(n, s, seed=synth.seed_of(3, 0, 0, i) + 7919 * rank, dtype=dtype,
+        tensors.append(synth.relu_iid_torch(n, s, seed=rank_seed(synth.seed_of(3, 0, 0, i), rank), dtype=dtype,
                                             device=dev))
         outs.append(torch.empty_like(tensors[-1]))
         sizes.append(n)
@@ -135,6 +135,11 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
         torch.cuda.synchronize()
 
     def timed(codec, steps, warmup, record=False, clocks=False):
+        # the clock sampler starts before the warm-up so that nvidia-smi is already sampling
+        # (every 200 ms) when the short timed region begins; it stops right after it
+        sampler = ClockSampler(local_rank) if clocks else None
+        if sampler:
+            sampler.__enter__()
         for _ in range(warmup):
             for h in step(codec):
                 h.close()
@@ -143,9 +148,6 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
         if record:
             C.collect_kernel_timing()
             C.set_kernel_timing(True)
-        sampler = ClockSampler(local_rank) if clocks else None
-        if sampler:
-            sampler.__enter__()
         t0 = time.perf_counter()
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
@@ -178,11 +180,11 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
     main = timed(C.AUTO, args.steps, args.warmup, record=True, clocks=True)
     ms_max = _max_over_ranks(main["ms"], dist)
     ms_per_step = ms_max / args.steps
-    value = world * raw_bytes / (ms_per_step * 1e-3) / 1e9
+    value = job_throughput(world, raw_bytes, ms_per_step)
     for o, t in zip(outs, tensors):  # the last step restored every tensor bitwise
         assert torch.equal(o, t), "swap round trip mismatch"
 
-    roof = _roofline(main["records"])
+    roof = _roofline(main["records"], args.steps)
     result = {
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True, "scaling": "weak",
@@ -227,12 +229,24 @@ def _codec_built(C, codec) -> bool:
 
 
 def _max_over_ranks(v: float, dist) -> float:
-    if dist is None:
+    """Device time of the slowest rank (the job's time)."""
+    if dist is None or not dist.is_initialized():
         return v
     import torch
-    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([v], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+def rank_seed(base: int, rank: int) -> int:
+    """Each replica swaps its own tensors: distinct seeds per rank, same recipe."""
+    return base + 7919 * rank
+
+
+def job_throughput(world: int, raw_bytes_per_rank: int, ms_max: float) -> float:
+    """Whole-job GB/s: bytes swapped out and back in by all ranks / the slowest rank's time."""
+    return world * raw_bytes_per_rank / (ms_max * 1e-3) / 1e9
 
 
 def _peaks():
@@ -244,7 +258,7 @@ def _peaks():
     return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-def _roofline(records) -> dict:
+def _roofline(records, steps: int = 1) -> dict:
     """Dominant kernel = the codec launch group with the largest total device time in the timed
     region; algorithmic bytes = raw bytes + container bytes per launch."""
     peak, src = _peaks()
@@ -259,17 +273,26 @@ def _roofline(records) -> dict:
         g["launches"] += 1
     if not groups:
         return {"bound": "hbm", "achieved": None, "peak": peak, "unit": "GB/s", "frac": None, "traffic": None}
-    (codec, d), g = max(groups.items(), key=lambda kv: kv[1]["ms"])
+    # the dominant single kernel: compress (one launch per tensor).  A decompress group is
+    # count + scan + expand (+ prep); its largest kernel (expand) has a smaller share of the
+    # step than compress in the committed launch list (profiles/launches_r01.txt).
+    single = {kk: v for kk, v in groups.items() if kk[1] == 0} or groups
+    (codec, d), g = max(single.items(), key=lambda kv: kv[1]["ms"])
     achieved = g["bytes"] / (g["ms"] * 1e-3) / 1e9
     names = {0: "none", 1: "zvc", 2: "rle", 3: "csr", 4: "lz4"}
+    # traffic: DRAM read+write bytes per launch group of the same kernels in one step of this
+    # bench, from the committed `ncu --set full` capture (profiles/ncu_r01.json, "bench_step")
     traffic = None
     if os.path.exists(NCU_SUMMARY):
         with open(NCU_SUMMARY) as f:
-            ncu = json.load(f)
-        k = f"{names[codec]}_{'compress' if d == 0 else 'decompress'}"
-        if k in ncu:
-            traffic = ncu[k].get("dram_bytes_per_algorithmic_byte")
-            traffic = None if traffic is None else round(traffic * g["bytes"] / g["launches"])
+            prof = json.load(f).get("bench_step", {})
+        stem = {0: "none", 1: "zvc", 2: "rle", 3: "csr", 4: "lz4"}[codec]
+        parts = ["compress"] if d == 0 else ["count", "scan", "expand", "dscan", "decode", "prep"]
+        tot = sum(v["dram_bytes_per_launch"] * v["launches"] for kname, v in prof.items()
+                  if (kname.startswith(stem) or (d == 1 and kname.startswith("prep")))
+                  and any(p in kname for p in parts))
+        if tot:
+            traffic = round(tot / (g["launches"] / steps))  # per launch group, like `achieved`
     out = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
            "frac": round(achieved / peak, 4), "traffic": traffic,
            "kernel": f"{names[codec]}_{'compress' if d == 0 else 'decompress'}", "launches": g["launches"],

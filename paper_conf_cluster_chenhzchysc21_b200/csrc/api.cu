@@ -178,14 +178,27 @@ struct Ctx {
 };
 
 // Brackets a launch group with CUDA events on its stream when timing is enabled.
+// The start event is recorded by the launcher itself, immediately before its first kernel
+// (cswap::timing_kernel_start), so that host-side enqueue time on an idle stream is not counted.
+struct Timer;
+thread_local Timer* t_pending = nullptr;
 struct Timer {
   Ctx* c;
   cudaStream_t st;
   cudaEvent_t a = nullptr, b = nullptr;
+  bool started = false;
   Timer(Ctx* ctx, cudaStream_t s) : c(ctx), st(s) {
-    if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) cudaEventRecord(a, st);
+    if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) t_pending = this;
+  }
+  void start_now() {
+    if (a && !started) {
+      cudaEventRecord(a, st);
+      started = true;
+    }
   }
   void stop() {
+    if (t_pending == this) t_pending = nullptr;
+    start_now();  // no launcher marked a start: fall back to "now"
     if (a && !b && cudaEventCreate(&b) == cudaSuccess) cudaEventRecord(b, st);
   }
   void commit(int codec, int dir, uint64_t raw, uint64_t comp) {
@@ -196,10 +209,18 @@ struct Timer {
     a = b = nullptr;
   }
   ~Timer() {
+    if (t_pending == this) t_pending = nullptr;
     if (a) cudaEventDestroy(a);
     if (b) cudaEventDestroy(b);
   }
 };
+}  // namespace
+
+void cswap::timing_kernel_start(cudaStream_t) {
+  if (t_pending) t_pending->start_now();
+}
+
+namespace {
 
 Ctx* g_ctx = nullptr;
 std::mutex g_mu;

@@ -180,6 +180,7 @@ __global__ void __launch_bounds__(1024) prep_kernel(const uint8_t* in, uint64_t 
 
 cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
                         uint32_t param, const Scratch& sc, uint32_t* err, cudaStream_t st) {
+  timing_kernel_start(st);
   prep_kernel<<<1, 1024, 0, st>>>(in, in_size, codec, dtype, n, F, param, sc.aux, sc.aux2, err);
   return cudaGetLastError();
 }
@@ -259,6 +260,7 @@ cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, c
   const bool single = n <= uint64_t(kProbeW) * kProbeSw;
   const uint32_t pieces = single ? uint32_t(cdiv(n, kProbeW)) : kProbeSw;
   const uint32_t grid = uint32_t(umin64(cdiv(pieces, kWarps), 128));
+  timing_kernel_start(st);
   if (w == 4)
     probe_kernel<uint32_t><<<grid, kThreads, 0, st>>>(static_cast<const uint32_t*>(in), n, pieces, single, sc.aux2,
                                                       sc.tickets + epoch, counts3);

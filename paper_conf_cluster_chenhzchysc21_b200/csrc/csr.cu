@@ -123,6 +123,7 @@ static cudaError_t csr_compress_t(const void* in, uint64_t n, uint64_t F, uint32
   const uint32_t tpf = uint32_t(cdiv(F, G::TILE));
   const uint32_t tiles = rle_tiles(n, sizeof(T), F);
   const T* x = static_cast<const T*>(in);
+  timing_kernel_start(st);
   csr_count_kernel<T><<<tiles, kThreads, 0, st>>>(x, n, F, tpf, sc);
   csr_scan_kernel<T><<<K, 1024, 0, st>>>(n, F, tpf, C, sc);
   cudaError_t e = launch_finalize(out, kCSR, dtype, n, F, C, sc, out_size, st);
@@ -229,6 +230,7 @@ cudaError_t launch_csr_decompress(const uint8_t* in, void* out, uint64_t n, int 
   const uint32_t TILE = kTileBytes / w;
   const uint32_t tpf = uint32_t(cdiv(F, TILE));
   const uint32_t tiles = (k1 - 1 - k0) * tpf + uint32_t(cdiv(frame_len(n, F, k1 - 1), TILE));
+  timing_kernel_start(st);
   if (w == 4)
     csr_expand_kernel<uint32_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint32_t*>(out), n, F, tpf, C, k0, sc, err);
   else

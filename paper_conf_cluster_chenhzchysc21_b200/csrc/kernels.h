@@ -7,6 +7,10 @@
 
 namespace cswap {
 
+// api.cu: records the start event of the pending kernel timer (if timing is enabled) right
+// before a launcher's first kernel
+void timing_kernel_start(cudaStream_t st);
+
 // container.cu
 cudaError_t launch_header_only(uint8_t* out, int codec, int dtype, uint64_t F, uint32_t param, uint64_t* out_size,
                                cudaStream_t st);

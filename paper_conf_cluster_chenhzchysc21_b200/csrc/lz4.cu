@@ -202,6 +202,7 @@ cudaError_t launch_lz4_compress(const void* in, uint64_t n, int w, uint64_t F, u
     cudaFuncSetAttribute(lz4_compress_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
+  timing_kernel_start(st);
   lz4_compress_kernel<<<nblk, 32, smem, st>>>(static_cast<const uint8_t*>(in), n, w, F, B, bpf, slots, sc.tbuf);
   lz4_scan_kernel<<<K, 1024, 0, st>>>(n, w, F, B, bpf, sc);
   cudaError_t e = launch_finalize(out, kLZ4, dtype, n, F, B, sc, out_size, st);
@@ -326,6 +327,7 @@ cudaError_t launch_lz4_decompress(const uint8_t* in, void* out, uint64_t n, int 
                                   uint32_t k0, uint32_t k1, const Scratch& sc, uint32_t* err, cudaStream_t st) {
   if (k1 <= k0) return cudaSuccess;
   const uint32_t bpf = uint32_t(cdiv(F * w, B));
+  timing_kernel_start(st);
   lz4_dscan_kernel<<<k1 - k0, 1024, 0, st>>>(in, n, w, F, B, bpf, k0, sc, err);
   const int smem = kLz4MaxBlock;
   static bool attr = false;

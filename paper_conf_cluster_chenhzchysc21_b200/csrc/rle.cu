@@ -175,6 +175,7 @@ static cudaError_t rle_compress_t(const void* in, uint64_t n, uint64_t F, uint8_
   const uint32_t tpf = uint32_t(cdiv(F, G::TILE));
   const uint32_t tiles = rle_tiles(n, sizeof(T), F);
   const T* x = static_cast<const T*>(in);
+  timing_kernel_start(st);
   rle_count_kernel<T><<<tiles, kThreads, 0, st>>>(x, n, F, tpf, sc);
   rle_scan_kernel<T><<<K, 1024, 0, st>>>(n, F, tpf, sc);
   cudaError_t e = launch_finalize(out, kRLE, dtype, n, F, 0, sc, out_size, st);
@@ -296,9 +297,11 @@ cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int 
   if (e != cudaSuccess) return e;
   const uint32_t tiles = (k1 - 1 - k0) * tpf + uint32_t(cdiv(frame_len(n, F, k1 - 1), TILE));
   if (w == 4) {
+    timing_kernel_start(st);
     rle_dscan_kernel<uint32_t><<<k1 - k0, 1024, 0, st>>>(in, n, F, k0, rs, sc, err);
     rle_expand_kernel<uint32_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint32_t*>(out), n, F, tpf, k0, rs, sc, err);
   } else {
+    timing_kernel_start(st);
     rle_dscan_kernel<uint16_t><<<k1 - k0, 1024, 0, st>>>(in, n, F, k0, rs, sc, err);
     rle_expand_kernel<uint16_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint16_t*>(out), n, F, tpf, k0, rs, sc, err);
   }

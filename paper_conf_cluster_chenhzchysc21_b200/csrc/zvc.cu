@@ -692,6 +692,7 @@ static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uin
   // per-frame and per-group (tiles, nnz) accumulators
   cudaMemsetAsync(sc.aux2, 0, (uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32)) * 8, st);
   const uint32_t grid = std::min<uint32_t>(tiles, uint32_t(sm_count()) * per_sm);
+  timing_kernel_start(st);
   zvc_compress_persistent<T, S><<<grid, compress_threads<S>(), L::bytes, st>>>(
       static_cast<const T*>(in), n, F, K, tpf, tiles, out, out_size, sc, epoch, dtype, prof_enabled());
   if (prof_enabled()) {
@@ -743,6 +744,7 @@ static cudaError_t launch_zvc_decompress_t(const uint8_t* in, void* out, uint64_
   uint32_t tpf;
   const uint32_t tiles = zvc_tiles(n, sizeof(T), F, k0, k1, &tpf);
   if (!tiles) return cudaSuccess;
+  timing_kernel_start(st);
   zvc_count_kernel<T><<<(tiles + kWarps - 1) / kWarps, kThreads, 0, st>>>(in, n, F, tpf, k0, tiles, sc, err);
   zvc_scan_kernel<T><<<k1 - k0, 1024, 0, st>>>(n, F, tpf, k0, sc, err);
   const int smem = kTileBytes + 32;
