@@ -297,14 +297,13 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
   // count(i) runs before emit(i-1), so a tile's count never waits for an older tile's offset.
   const uint32_t lt = (1u << lane) - 1u;
   constexpr uint32_t SLAB = G::PER_WARP * G::W;  // bytes per slab (4 KiB)
-  auto load_row = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t q, uint32_t te, uint32_t be) {
+  // element e of the tile: from the stage (bulk-copied part), the global tail, or zero
+  auto load_elem = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t e, uint32_t te, uint32_t be) {
     constexpr bool full = decltype(full_tag)::value;
-    if (full) return reinterpret_cast<const uint32_t*>(stage)[q];
-    if (sizeof(T) == 4) return q < be ? reinterpret_cast<const uint32_t*>(stage)[q] : (q < te ? uint32_t(gsrc[q]) : 0u);
-    const uint32_t e = 2 * q;
-    if (e + 2 <= be) return reinterpret_cast<const uint32_t*>(stage)[q];
-    return (e < te ? uint32_t(gsrc[e]) : 0u) | ((e + 1 < te ? uint32_t(gsrc[e + 1]) : 0u) << 16);
+    if (full) return uint32_t(reinterpret_cast<const T*>(stage)[e]);
+    return e < be ? uint32_t(reinterpret_cast<const T*>(stage)[e]) : (e < te ? uint32_t(gsrc[e]) : 0u);
   };
+  constexpr int EROWS = G::PER_WARP / 32;  // rows of 32 elements per slab (32 fp32 / 64 fp16)
   auto group_wait = [&](uint64_t* bar, uint32_t parity) {  // one warp polls, the rest block in bar.sync
     if (warp == 0) mbar_wait(bar, parity);
     consumer_sync();
@@ -313,47 +312,28 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
 
   auto count_slab = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be,
                         uint32_t* bm_out) {
-    const uint32_t q0 = warp * (SLAB / 4);
+    // row m = elements [32m, 32m+32) of the slab: one ballot is bitmap word (slab word m)
+    const uint32_t e0 = warp * G::PER_WARP + lane;
     uint32_t tot = 0;
 #pragma unroll 8
-    for (int m = 0; m < ROWS; m++) {
-      const uint32_t v = load_row(full_tag, stage, gsrc, q0 + 32 * m + lane, te, be);
-      if (sizeof(T) == 4) {
-        const uint32_t w = __ballot_sync(0xffffffffu, v != 0);
-        if (lane == 0) bm_out[m] = w;
-        tot += __popc(w);
-      } else {
-        const uint32_t lo = __ballot_sync(0xffffffffu, (v & 0xFFFFu) != 0);
-        const uint32_t hi = __ballot_sync(0xffffffffu, (v >> 16) != 0);
-        if (lane == 0) {
-          bm_out[2 * m] = spread16(lo) | (spread16(hi) << 1);
-          bm_out[2 * m + 1] = spread16(lo >> 16) | (spread16(hi >> 16) << 1);
-        }
-        tot += __popc(lo) + __popc(hi);
-      }
+    for (int m = 0; m < EROWS; m++) {
+      const uint32_t v = load_elem(full_tag, stage, gsrc, e0 + 32 * m, te, be);
+      const uint32_t w = __ballot_sync(0xffffffffu, v != 0);
+      if (lane == 0) bm_out[m] = w;
+      tot += __popc(w);
     }
     return tot;
   };
 
   auto emit_slab = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be, uint8_t* dst) {
-    const uint32_t q0 = warp * (SLAB / 4);
+    const uint32_t e0 = warp * G::PER_WARP + lane;
     uint32_t pre = 0;
 #pragma unroll 8
-    for (int m = 0; m < ROWS; m++) {
-      const uint32_t v = load_row(full_tag, stage, gsrc, q0 + 32 * m + lane, te, be);
-      if (sizeof(T) == 4) {
-        const uint32_t w = __ballot_sync(0xffffffffu, v != 0);
-        if (v) reinterpret_cast<uint32_t*>(dst)[pre + __popc(w & lt)] = v;
-        pre += __popc(w);
-      } else {
-        const uint32_t lo = __ballot_sync(0xffffffffu, (v & 0xFFFFu) != 0);
-        const uint32_t hi = __ballot_sync(0xffffffffu, (v >> 16) != 0);
-        uint32_t r = pre + __popc(lo & lt) + __popc(hi & lt);
-        uint16_t* d16 = reinterpret_cast<uint16_t*>(dst);
-        if (v & 0xFFFFu) d16[r++] = uint16_t(v);
-        if (v >> 16) d16[r] = uint16_t(v >> 16);
-        pre += __popc(lo) + __popc(hi);
-      }
+    for (int m = 0; m < EROWS; m++) {
+      const uint32_t v = load_elem(full_tag, stage, gsrc, e0 + 32 * m, te, be);
+      const uint32_t w = __ballot_sync(0xffffffffu, v != 0);
+      if (v) reinterpret_cast<T*>(dst)[pre + __popc(w & lt)] = T(v);
+      pre += __popc(w);
     }
   };
 
@@ -555,18 +535,23 @@ __global__ void __launch_bounds__(kThreads) zvc_expand_kernel(const uint8_t* __r
   const uint64_t fstart = sc.aux[k], fend = fstart + sc.aux2[k];
   const uint64_t vbeg = sc.tbuf[t];
   const uint64_t vend = (j + 1 < uint32_t(cdiv(Fk, G::TILE))) ? sc.tbuf[t + 1] : 0;  // next tile's start
-  if (tid == 0) {
-    mbar_init(&s_bar, 1);
-  }
-  __syncthreads();
-  // tile value count = popcount of the bitmap slice; the span end for the last tile of the
-  // frame comes from the count, for others from the next tile's offset
+  // Both bulk copies are issued at once (one round trip): the bitmap slice, and the value span
+  // known from the scanned offsets alone — [this tile's offset, next tile's offset), or up to
+  // the frame end for the frame's last tile (an aligned superset inside the container).
   const uint32_t bm_bytes = ((nw * 4) + 15) & ~15u;
   const uint8_t* bsrc = in + fstart + uint64_t(j) * G::WT * 4;
+  const uint64_t abeg = vbeg & ~uint64_t(15);
+  const uint64_t aend = vend ? a16(vend) : fend;
+  const uint32_t d = uint32_t(vbeg - abeg);
+  const bool span_ok = vbeg >= fstart && aend <= fend && aend >= abeg && aend - abeg <= kTileBytes + 32;
   if (tid == 0) {
-    mbar_expect_tx(&s_bar, bm_bytes);
+    mbar_init(&s_bar, 1);
+    const uint32_t vbytes = span_ok ? uint32_t(aend - abeg) : 0;
+    mbar_expect_tx(&s_bar, bm_bytes + vbytes);
     bulk_g2s(s_bm, bsrc, bm_bytes, &s_bar);
+    if (vbytes) bulk_g2s(s_val, in + abeg, vbytes, &s_bar);
   }
+  __syncthreads();
   mbar_wait(&s_bar, 0);
   // per-warp totals
   {
@@ -590,20 +575,8 @@ __global__ void __launch_bounds__(kThreads) zvc_expand_kernel(const uint8_t* __r
     nnz += s_woff[w];
   }
   const uint64_t vlast = vbeg + uint64_t(nnz) * G::W;
-  const uint64_t abeg = vbeg & ~uint64_t(15), aend = a16(vlast);
-  const uint32_t d = uint32_t(vbeg - abeg);
-  const bool ok = aend <= fend && vbeg >= fstart && (vend == 0 || vend == vlast);
-  if (tid == 0) {
-    if (!ok) set_error(err, kErrCorrupt);
-    const uint32_t bytes = ok ? uint32_t(aend - abeg) : 0;
-    if (bytes) {
-      mbar_expect_tx(&s_bar, bytes);
-      bulk_g2s(s_val, in + abeg, bytes, &s_bar);
-    } else {
-      mbar_arrive(&s_bar);
-    }
-  }
-  mbar_wait(&s_bar, 1);
+  const bool ok = span_ok && (vend ? vend == vlast : a16(vlast) <= fend);
+  if (!ok && tid == 0) set_error(err, kErrCorrupt);
   T* dst = outp + uint64_t(k) * F + uint64_t(j) * G::TILE;
   uint32_t r = woff;
 #pragma unroll
