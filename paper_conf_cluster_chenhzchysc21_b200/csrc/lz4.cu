@@ -8,16 +8,16 @@
 // (MINMATCH 4, MFLIMIT 12, LASTLITERALS 5, HASHLOG 12, lookup-then-insert at every scanned
 // position, nothing inserted inside matches).  Frame: u32 csize[nblk] pad16 | blocks | pad16.
 //
-// Compress: one warp per block, block + 4096-entry u16 hash table in shared memory.  The warp
-// scans 32 consecutive positions at a time: lane j's candidate is the latest earlier lane with the
-// same hash (__match_any_sync) else the table entry; the first lane whose candidate verifies ends
-// the batch; lanes up to it insert (latest lane per hash wins).  This is exactly the sequential
-// parse.  Matches are extended 32 bytes per step; sequences are written by the
-// whole warp into a per-block scratch slot.  Then: per-frame scan of block sizes -> frame table
-// -> pack (one CTA per block).
-// Decompress: per-frame scan of csize -> block offsets; one warp per block decodes into shared
-// memory (literal and match copies 32 bytes per step, short-offset matches by pattern
-// replication) with every read and write bounds-checked, then stores the block with 16-byte stores.
+// Compress: one warp per block (4 per CTA), the 4096-entry u16 hash table in shared memory, the
+// block read through L1/L2.  The warp scans 32 consecutive positions at a time: lane j's
+// candidate is the latest earlier lane with the same hash (__match_any_sync) else the table
+// entry; the first lane whose candidate verifies ends the batch; lanes up to it insert (latest
+// lane per hash wins).  This is exactly the sequential parse.  Matches are
+// extended 32 bytes per step; sequences are written by the whole warp into a per-block scratch
+// slot.  Then: per-frame scan of block sizes -> frame table -> pack (one CTA per block).
+// Decompress: per-frame scan of csize -> block offsets; one warp per block decodes straight into
+// the output (literal and match copies 32 bytes per step, short-offset matches by shuffling the
+// `offset`-byte pattern) with every read and write bounds-checked.
 #include "kernels.h"
 #include "tile_common.cuh"
 
@@ -69,23 +69,29 @@ __device__ __forceinline__ uint32_t emit_seq(uint8_t* out, uint32_t op, const ui
 
 // one warp per block; blocks indexed globally (frame-major), block b of frame k covers bytes
 // [b*B, min((b+1)*B, Fk*w)) of the frame
-__global__ void __launch_bounds__(32) lz4_compress_kernel(const uint8_t* __restrict__ in, uint64_t n, int w,
-                                                          uint64_t F, uint32_t B, uint32_t bpf, uint8_t* slots,
-                                                          uint64_t* csize) {
-  extern __shared__ __align__(16) uint8_t smem[];
-  uint8_t* s_src = smem;                                              // B + 16 bytes
-  uint16_t* s_tab = reinterpret_cast<uint16_t*>(smem + kLz4MaxBlock + 16);  // 4096 entries
-  const int lane = threadIdx.x;
-  const uint32_t blk = blockIdx.x;
+// The source block is read through L1/L2 (it is not staged): only the 8 KiB hash table lives in
+// shared memory, so 4 blocks per CTA and ~28 parsing warps per SM hide each other's latency
+// (staging the 64 KiB block limited an SM to 3 warps: 7.6 GB/s at s = 0.5).
+constexpr int kLz4Warps = 4;
+
+__device__ __forceinline__ uint32_t le32_g(const uint8_t* s, uint32_t p) {  // s 16-aligned; p+8 <= block end
+  const uint32_t* w = reinterpret_cast<const uint32_t*>(s);
+  const uint32_t a = __ldg(w + (p >> 2)), b = __ldg(w + (p >> 2) + 1);
+  return __funnelshift_r(a, b, (p & 3) * 8);
+}
+
+__global__ void __launch_bounds__(32 * kLz4Warps) lz4_compress_kernel(const uint8_t* __restrict__ in, uint64_t n,
+                                                                      int w, uint64_t F, uint32_t B, uint32_t bpf,
+                                                                      uint32_t nblk, uint8_t* slots, uint64_t* csize) {
+  __shared__ uint16_t s_tabs[kLz4Warps][4096];
+  const int lane = threadIdx.x & 31;
+  const uint32_t blk = blockIdx.x * kLz4Warps + (threadIdx.x >> 5);
+  if (blk >= nblk) return;
+  uint16_t* s_tab = s_tabs[threadIdx.x >> 5];
   const uint32_t k = blk / bpf, b = blk % bpf;
   const uint64_t fbytes = frame_len(n, F, k) * uint64_t(w);
   const uint32_t L = uint32_t(umin64(B, fbytes - uint64_t(b) * B));
-  const uint8_t* src = in + uint64_t(k) * F * w + uint64_t(b) * B;
-  // stage the block (16-byte vectors; B and every block start are 16-aligned, the tail is scalar)
-  const uint32_t nv = L / 16;
-  for (uint32_t v = lane; v < nv; v += 32)
-    reinterpret_cast<uint4*>(s_src)[v] = ldg_stream(reinterpret_cast<const uint4*>(src) + v);
-  for (uint32_t q = nv * 16 + lane; q < L + 16; q += 32) s_src[q] = q < L ? src[q] : 0;
+  const uint8_t* s_src = in + uint64_t(k) * F * w + uint64_t(b) * B;  // global, read-only
   for (uint32_t h = lane; h < 4096; h += 32) s_tab[h] = kLz4Empty;
   __syncwarp();
   uint8_t* out = slots + uint64_t(blk) * kLz4SlotBytes;
@@ -96,13 +102,13 @@ __global__ void __launch_bounds__(32) lz4_compress_kernel(const uint8_t* __restr
     while (i <= limit) {
       const uint32_t pos = i + lane;
       const bool active = pos <= limit;
-      const uint32_t v = active ? le32_smem(s_src, pos) : 0;
+      const uint32_t v = active ? le32_g(s_src, pos) : 0;
       const uint32_t h = active ? (v * 2654435761u) >> 20 : 0x10000u + lane;
       const uint32_t same = __match_any_sync(0xffffffffu, h);
       const uint32_t earlier = same & lt;
       uint32_t cand = kLz4Empty;
       if (active) cand = earlier ? i + (31 - __clz(earlier)) : s_tab[h];
-      const bool ok = active && cand != kLz4Empty && le32_smem(s_src, cand) == v;
+      const bool ok = active && cand != kLz4Empty && le32_g(s_src, cand) == v;
       const uint32_t mm = __ballot_sync(0xffffffffu, ok);
       // lanes that insert: up to the first matching lane (all active lanes if none matched);
       // within a hash group the latest inserting lane wins
@@ -196,14 +202,9 @@ cudaError_t launch_lz4_compress(const void* in, uint64_t n, int w, uint64_t F, u
   const uint32_t K = uint32_t(cdiv(n, F));
   uint32_t bpf;
   const uint32_t nblk = lz4_blocks(n, w, F, B, &bpf);
-  const int smem = kLz4MaxBlock + 16 + 4096 * 2;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(lz4_compress_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    attr = true;
-  }
   timing_kernel_start(st);
-  lz4_compress_kernel<<<nblk, 32, smem, st>>>(static_cast<const uint8_t*>(in), n, w, F, B, bpf, slots, sc.tbuf);
+  lz4_compress_kernel<<<(nblk + kLz4Warps - 1) / kLz4Warps, 32 * kLz4Warps, 0, st>>>(
+      static_cast<const uint8_t*>(in), n, w, F, B, bpf, nblk, slots, sc.tbuf);
   lz4_scan_kernel<<<K, 1024, 0, st>>>(n, w, F, B, bpf, sc);
   cudaError_t e = launch_finalize(out, kLZ4, dtype, n, F, B, sc, out_size, st);
   if (e != cudaSuccess) return e;
@@ -245,13 +246,24 @@ __global__ void __launch_bounds__(1024) lz4_dscan_kernel(const uint8_t* __restri
   if (threadIdx.x == 0 && a16(4ull * nb) + a16(carry) != fb) set_error(err, kErrCorrupt);
 }
 
-__global__ void __launch_bounds__(32) lz4_decode_kernel(const uint8_t* __restrict__ in, uint8_t* __restrict__ outp,
-                                                        uint64_t n, int w, uint64_t F, uint32_t B, uint32_t bpf,
-                                                        uint32_t k0, Scratch sc, uint32_t* err) {
-  extern __shared__ __align__(16) uint8_t s_out[];  // B bytes
+// One warp per block, writing straight into the output tensor (no shared-memory staging, so
+// ~16 warps per SM); match sources are read back with ld.global.cg (L2, coherent with the
+// warp's own earlier stores after __syncwarp).
+__device__ __forceinline__ uint8_t ld_cg_u8(const uint8_t* p) {
+  uint16_t v;
+  asm volatile("ld.global.cg.u8 %0, [%1];" : "=h"(v) : "l"(p) : "memory");
+  return uint8_t(v);
+}
+
+__global__ void __launch_bounds__(32 * kLz4Warps) lz4_decode_kernel(const uint8_t* __restrict__ in, uint8_t* outp,
+                                                                    uint64_t n, int w, uint64_t F, uint32_t B,
+                                                                    uint32_t bpf, uint32_t k0, uint32_t nslots,
+                                                                    Scratch sc, uint32_t* err) {
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
-  const int lane = threadIdx.x;
-  const uint32_t k = k0 + blockIdx.x / bpf, b = blockIdx.x % bpf;
+  const int lane = threadIdx.x & 31;
+  const uint32_t slot = blockIdx.x * kLz4Warps + (threadIdx.x >> 5);
+  if (slot >= nslots) return;
+  const uint32_t k = k0 + slot / bpf, b = slot % bpf;
   const uint64_t fbytes = frame_len(n, F, k) * uint64_t(w);
   const uint32_t nb = uint32_t(cdiv(fbytes, B));
   if (b >= nb) return;
@@ -262,9 +274,10 @@ __global__ void __launch_bounds__(32) lz4_decode_kernel(const uint8_t* __restric
   const uint64_t start = a16(4ull * nb) + sc.tbuf2[blk];
   bool bad = start + cs > fb;
   const uint8_t* ip0 = in + fstart + start;
+  uint8_t* dst = outp + uint64_t(k) * F * w + uint64_t(b) * B;
   uint64_t ip = 0;
   uint32_t op = 0;
-  auto rd = [&](uint64_t at) -> uint32_t { return at < cs ? ip0[at] : 0u; };
+  auto rd = [&](uint64_t at) -> uint32_t { return at < cs ? __ldg(ip0 + at) : 0u; };
   while (!bad) {
     if (ip >= cs) { bad = true; break; }
     const uint32_t token = rd(ip++);
@@ -279,10 +292,9 @@ __global__ void __launch_bounds__(32) lz4_decode_kernel(const uint8_t* __restric
       if (bad) break;
     }
     if (ip + nlit > cs || op + nlit > L) { bad = true; break; }
-    for (uint32_t q = lane; q < nlit; q += 32) s_out[op + q] = ip0[ip + q];
+    for (uint32_t q = lane; q < nlit; q += 32) dst[op + q] = __ldg(ip0 + ip + q);
     ip += nlit;
     op += nlit;
-    __syncwarp();
     if (ip == cs) break;  // last sequence: literals only
     if (ip + 2 > cs) { bad = true; break; }
     const uint32_t offset = rd(ip) | (rd(ip + 1) << 8);
@@ -299,28 +311,26 @@ __global__ void __launch_bounds__(32) lz4_decode_kernel(const uint8_t* __restric
     }
     mlen += 4;
     if (offset == 0 || offset > op || op + mlen > L) { bad = true; break; }
+    __syncwarp();  // the match source may have been written by other lanes
     if (offset >= 32) {  // non-overlapping within a 32-byte step
       for (uint32_t q = 0; q < mlen; q += 32) {
-        if (q + lane < mlen) s_out[op + q + lane] = s_out[op + q + lane - offset];
+        if (q + lane < mlen) dst[op + q + lane] = ld_cg_u8(dst + op + q + lane - offset);
         __syncwarp();
       }
     } else {  // short offset: the match repeats the last `offset` bytes
       const uint32_t base = op - offset;
-      for (uint32_t q = lane; q < mlen; q += 32) s_out[op + q] = s_out[base + (q % offset)];
+      const uint32_t pat = lane < int(offset) ? ld_cg_u8(dst + base + lane) : 0u;
+      for (uint32_t q0 = 0; q0 < mlen; q0 += 32) {  // whole-warp iterations: every lane shuffles
+        const uint32_t q = q0 + lane;
+        const uint32_t v = __shfl_sync(0xffffffffu, pat, q % offset);
+        if (q < mlen) dst[op + q] = uint8_t(v);
+      }
     }
     op += mlen;
     __syncwarp();
   }
   if (!bad && op != L) bad = true;
-  if (__any_sync(0xffffffffu, bad)) {
-    if (lane == 0) set_error(err, kErrCorrupt);
-    return;
-  }
-  __syncwarp();
-  uint8_t* dst = outp + uint64_t(k) * F * w + uint64_t(b) * B;
-  const uint32_t nv = L / 16;
-  for (uint32_t v = lane; v < nv; v += 32) stg_stream(reinterpret_cast<uint4*>(dst) + v, reinterpret_cast<const uint4*>(s_out)[v]);
-  for (uint32_t q = nv * 16 + lane; q < L; q += 32) dst[q] = s_out[q];
+  if (__any_sync(0xffffffffu, bad) && lane == 0) set_error(err, kErrCorrupt);
 }
 
 cudaError_t launch_lz4_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t B,
@@ -329,13 +339,9 @@ cudaError_t launch_lz4_decompress(const uint8_t* in, void* out, uint64_t n, int 
   const uint32_t bpf = uint32_t(cdiv(F * w, B));
   timing_kernel_start(st);
   lz4_dscan_kernel<<<k1 - k0, 1024, 0, st>>>(in, n, w, F, B, bpf, k0, sc, err);
-  const int smem = kLz4MaxBlock;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(lz4_decode_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    attr = true;
-  }
-  lz4_decode_kernel<<<(k1 - k0) * bpf, 32, B, st>>>(in, static_cast<uint8_t*>(out), n, w, F, B, bpf, k0, sc, err);
+  const uint32_t nslots = (k1 - k0) * bpf;
+  lz4_decode_kernel<<<(nslots + kLz4Warps - 1) / kLz4Warps, 32 * kLz4Warps, 0, st>>>(
+      in, static_cast<uint8_t*>(out), n, w, F, B, bpf, k0, nslots, sc, err);
   return cudaGetLastError();
 }
 
