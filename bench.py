@@ -331,8 +331,8 @@ def _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, r
     link = _link(torch)
     ex["link"] = link
     steps_b = max(2, min(args.steps, 3))
-    none = timed(C.NONE, steps_b, 1)
-    sc = timed(C.ZVC, steps_b, 1)
+    none = timed(C.NONE, steps_b, 3)
+    sc = timed(C.ZVC, steps_b, 3)
     ex["latency_ms"] = {"auto": main["ms"] / args.steps, "vdnn_none": none["ms"] / steps_b,
                         "sc_always_zvc": sc["ms"] / steps_b}
     comp = sum(q["bytes"] for q in main["handles"])
@@ -362,7 +362,100 @@ def _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, r
         per.append(row)
     ex["per_tensor"] = per
     ex["every_compressed_tensor_faster"] = all(r["chosen_ms"] < r["none_ms"] for r in per if r["codec"] != "none")
+    # decision accuracy (PAPER.md:305 analogue): the selector's codec vs the measured-fastest of
+    # the five choices, per tensor, on the workload set and on a mixed set whose sparsity
+    # structure makes every codec the right answer somewhere
+    ex["decision_accuracy"] = {
+        "workload": _decision_accuracy(C, torch, list(zip(tensors, outs, sizes)), dtype,
+                                       [r["codec"] for r in per]),
+        "mixed_set": _decision_accuracy(C, torch, _mixed_set(torch), None, None),
+    }
+    # overheads: probe kernel + readback, host selector
+    tp = []
+    for t, n in zip(tensors, sizes):
+        t0 = time.perf_counter()
+        pr = C.probe(t, n, dtype)
+        t1 = time.perf_counter()
+        C.select_from_probe(n, dtype, pr)
+        t2 = time.perf_counter()
+        tp.append((t1 - t0, t2 - t1))
+    ex["overheads_us"] = {"probe_incl_readback": round(1e6 * sum(a for a, _ in tp) / len(tp), 2),
+                          "select_host": round(1e6 * sum(b for _, b in tp) / len(tp), 2)}
     return ex
+
+
+def _swap_ms(C, torch, t, o, n, dtype, codec, reps=2):
+    """Best-of-reps device time of one swap out + swap in of a single tensor; returns
+    (ms, codec actually used)."""
+    stream = torch.cuda.current_stream()
+    best, used = 1e9, codec
+    for _ in range(reps):
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        h = C.swap_out(t, n, dtype, codec)
+        h.swap_in(o)
+        b.record(stream)
+        b.synchronize()
+        used = h.query()["codec"]
+        h.close()
+        best = min(best, a.elapsed_time(b))
+    return best, used
+
+
+def _mixed_set(torch):
+    """32 MiB tensors (f32 unless noted) spanning the sparsity structures of DESIGN.md §5:
+    iid ReLU masks, clustered zero runs, dead channels, a constant non-zero tensor, f16."""
+    import numpy as np
+
+    import synth
+    n = 8 << 20
+    specs = [("iid", s) for s in (0.0, 0.3, 0.6, 0.9, 0.99)] + \
+            [("clustered", s) for s in (0.5, 0.9, 0.99)] + [("dead", s) for s in (0.3, 0.8)] + \
+            [("constant", 0.0), ("iid_f16", 0.7)]
+    out = []
+    for i, (kind, s) in enumerate(specs):
+        seed = synth.seed_of(5, 0, 0, i)
+        dt = synth.F32
+        if kind == "iid":
+            x = synth.relu_iid(n, s, seed)
+        elif kind == "clustered":
+            x = synth.relu_clustered(n, s, 512, seed)
+        elif kind == "dead":
+            x = synth.channel_dead((64, 128, 32, 32), s, seed)
+        elif kind == "constant":
+            x = synth.constant(n, 0x3F800000)
+        else:
+            dt = synth.F16
+            x = synth.relu_iid(2 * n, s, seed, dtype=dt)
+        t = torch.from_numpy(x.view(np.int32 if dt == synth.F32 else np.int16)).cuda()
+        out.append((t, torch.empty_like(t), x.size, dt, f"{kind}_{s}"))
+    return out
+
+
+def _decision_accuracy(C, torch, items, dtype, chosen) -> dict:
+    """Selector's codec (AUTO) vs the measured-fastest codec per tensor. A choice within 2 % of
+    the fastest also counts as correct (`within_2pct`): the cost model cannot separate those."""
+    rows, exact, near = [], 0, 0
+    for i, it in enumerate(items):
+        if dtype is None:
+            t, o, n, dt, label = it
+        else:
+            (t, o, n), dt, label = it, dtype, str(i)
+        times = {C.CODEC_NAMES[c]: round(_swap_ms(C, torch, t, o, n, dt, c)[0], 4)
+                 for c in (C.NONE, C.ZVC, C.RLE, C.CSR, C.LZ4)}
+        if chosen is None:
+            ms_auto, used = _swap_ms(C, torch, t, o, n, dt, C.AUTO, reps=1)
+            pick = C.CODEC_NAMES[used]
+        else:
+            pick = chosen[i]
+        fastest = min(times, key=times.get)
+        exact += pick == fastest
+        near += times[pick] <= 1.02 * times[fastest]
+        rows.append({"tensor": label, "chosen": pick, "fastest": fastest, "ms": times})
+    k = len(rows)
+    return {"exact": exact, "within_2pct": near, "total": k, "frac": round(exact / k, 4),
+            "frac_within_2pct": round(near / k, 4), "per_tensor": rows}
 
 
 def _e2e(args, C, torch, tensors, outs, sizes, dtype, w, dist, world, stream) -> dict:
