@@ -273,10 +273,11 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
 // on the stream when the lease ends.
 struct Lease {
   Block* b = nullptr;
+  Ctx* ctx = nullptr;
   cudaStream_t st = nullptr;
   std::unique_lock<std::mutex> lk;
   cswap_status status = CSWAP_OK;
-  Lease(Ctx& c, cudaStream_t s, uint64_t tiles, uint64_t aux) : st(s) {
+  Lease(Ctx& c, cudaStream_t s, uint64_t tiles, uint64_t aux) : ctx(&c), st(s) {
     const uint32_t start = c.rr.fetch_add(1);
     for (int i = 0; i < kBlocks && !b; i++) {
       Block& cand = c.blocks[(start + i) % kBlocks];
@@ -296,9 +297,10 @@ struct Lease {
   }
   uint32_t epoch() {
     if (++b->epoch >= kEpochs) {
-      cudaMemsetAsync(b->sc.status, 0, b->sc.cap_tiles * 8, st);
-      cudaMemsetAsync(b->sc.tickets, 0, kEpochs * 4, st);
-      cudaMemsetAsync(b->sc.aux, 0, b->sc.cap_aux * 8, st);  // epoch-tagged frame starts
+      launch_zero_words(b->sc.status, b->sc.cap_tiles * 2, st);
+      launch_zero_words(b->sc.tickets, kEpochs, st);
+      launch_zero_words(b->sc.aux, b->sc.cap_aux * 2, st);  // epoch-tagged frame starts
+      ctx->launches += 3;
       b->epoch = 1;
     }
     return b->epoch;
@@ -379,11 +381,11 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       c->launches++;
       return cuda_status(launch_none_compress(in, n, w, F, dtype, out, out_size, st), "none_compress");
     case CSWAP_CODEC_ZVC: {
-      uint32_t tpf = 0;
-      const uint32_t tiles = zvc_tiles(n, w, F, 0, K, &tpf);
-      Lease L(*c, st, tiles, uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32) + 2);
+      uint64_t tiles = 0, aux = 0;
+      zvc_compress_scratch(n, w, F, &tiles, &aux);
+      Lease L(*c, st, tiles, aux);
       TRY(L.status);
-      c->launches++;
+      c->launches += 2;  // accumulator zero fill + persistent compress
       return cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, L.b->sc, L.epoch(), dtype, st), "zvc_compress");
     }
     case CSWAP_CODEC_RLE: {
@@ -427,7 +429,7 @@ cswap_status decompress_range(Ctx* c, Lease& L, const uint8_t* in, void* out, ui
   switch (codec) {
     case CSWAP_CODEC_NONE: return CSWAP_OK;  // handled by the caller (raw copy)
     case CSWAP_CODEC_ZVC:
-      c->launches++;
+      c->launches += 3;  // count, scan, expand
       return cuda_status(launch_zvc_decompress(in, out, n, w, F, k0, k1, L.b->sc, L.epoch(), err, st), "zvc_decompress");
     case CSWAP_CODEC_RLE:
       c->launches += 2;
@@ -647,10 +649,9 @@ cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uin
   // kernels flag errors in the lease's device word (never in host-mapped memory: every CTA
   // reads it); the word is merged into the caller's at the end
   uint32_t* e = L.b->sc.err;
-  CU(cudaMemsetAsync(e, 0, 4, st));
   const uint8_t* inb = static_cast<const uint8_t*>(in);
   c->launches += 2;
-  TRY(cuda_status(launch_prep(inb, in_size, codec, dtype, n, F, param_of(codec, f), L.b->sc, e, st), "prep"));
+  TRY(cuda_status(launch_prep(inb, in_size, codec, dtype, n, F, param_of(codec, f), L.b->sc, e, true, st), "prep"));
   cswap_status s = CSWAP_OK;
   if (n != 0) {
     if (codec == CSWAP_CODEC_NONE) {
@@ -895,7 +896,6 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
     Lease L(*c, st, decompress_tiles(n, w, f), decompress_aux(n, w, f));
     s = L.status;
     uint32_t* e_dev = L.b->sc.err;  // device word; merged into the handle's pinned slot at the end
-    if (s == CSWAP_OK && cudaMemsetAsync(e_dev, 0, 4, st) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "memset");
     uint64_t off = 0;
     for (uint32_t k0 = 0; k0 < K && s == CSWAP_OK; k0 += fpg) {
       const uint32_t k1 = std::min(K, k0 + fpg);
@@ -917,7 +917,7 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
       if (k0 == 0) {
         c->launches++;
         s = cuda_status(launch_prep(staging, h->bytes, h->codec, h->dtype, n, F, param_of(h->codec, f), L.b->sc,
-                                    e_dev, st),
+                                    e_dev, true, st),
                         "prep");
       }
       if (s == CSWAP_OK) s = decompress_range(c, L, staging, d_out, n, h->dtype, h->codec, f, k0, k1, e_dev, st);

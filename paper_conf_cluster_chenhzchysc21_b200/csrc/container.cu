@@ -98,6 +98,20 @@ cudaError_t launch_finalize(uint8_t* out, int codec, int dtype, uint64_t n, uint
   return cudaGetLastError();
 }
 
+// ---- zero fill of small scratch arrays (kept off the copy engines: a cudaMemsetAsync may be
+// queued behind a long D2H/H2D on the same engine) --------------------------------------------
+__global__ void zero_words_kernel(uint32_t* p, uint64_t words) {
+  for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < words; i += uint64_t(gridDim.x) * blockDim.x)
+    p[i] = 0u;
+}
+
+cudaError_t launch_zero_words(void* p, uint64_t words, cudaStream_t st) {
+  if (!words) return cudaSuccess;
+  const uint64_t blocks = std::min<uint64_t>((words + 255) / 256, 1184);
+  zero_words_kernel<<<unsigned(blocks), 256, 0, st>>>(static_cast<uint32_t*>(p), words);
+  return cudaGetLastError();
+}
+
 // ---- error word merge (device scratch word -> caller's word, first error wins) ---------------
 __global__ void err_merge_kernel(const uint32_t* src, uint32_t* dst) {
   const uint32_t v = *src;
@@ -138,12 +152,13 @@ __device__ __forceinline__ uint64_t block_excl_scan_u64(uint64_t v, uint64_t* s_
 
 __global__ void __launch_bounds__(1024) prep_kernel(const uint8_t* in, uint64_t in_size, int codec, int dtype,
                                                     uint64_t n, uint64_t F, uint32_t param, uint64_t* fstart,
-                                                    uint64_t* fbytes, uint32_t* err) {
+                                                    uint64_t* fbytes, uint32_t* err, int reset_err) {
   __shared__ int s_ok;
   __shared__ uint64_t s_total;
   __shared__ uint64_t s_warp[33];
   const uint32_t K = uint32_t(cdiv(n, F));
   if (threadIdx.x == 0) {
+    if (reset_err) *err = 0;  // first kernel of the decode: clears the lease's error word
     int ok = in_size >= 64;
     if (ok) {
       const uint32_t* h32 = reinterpret_cast<const uint32_t*>(in);
@@ -179,9 +194,9 @@ __global__ void __launch_bounds__(1024) prep_kernel(const uint8_t* in, uint64_t 
 }
 
 cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
-                        uint32_t param, const Scratch& sc, uint32_t* err, cudaStream_t st) {
+                        uint32_t param, const Scratch& sc, uint32_t* err, bool reset_err, cudaStream_t st) {
   timing_kernel_start(st);
-  prep_kernel<<<1, 1024, 0, st>>>(in, in_size, codec, dtype, n, F, param, sc.aux, sc.aux2, err);
+  prep_kernel<<<1, 1024, 0, st>>>(in, in_size, codec, dtype, n, F, param, sc.aux, sc.aux2, err, reset_err ? 1 : 0);
   return cudaGetLastError();
 }
 

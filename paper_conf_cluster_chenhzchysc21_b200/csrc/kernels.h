@@ -15,7 +15,9 @@ void timing_kernel_start(cudaStream_t st);
 cudaError_t launch_header_only(uint8_t* out, int codec, int dtype, uint64_t F, uint32_t param, uint64_t* out_size,
                                cudaStream_t st);
 cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
-                        uint32_t param, const Scratch& sc, uint32_t* err, cudaStream_t st);
+                        uint32_t param, const Scratch& sc, uint32_t* err, bool reset_err, cudaStream_t st);
+// zero `words` u32 words with a kernel (not the copy engine)
+cudaError_t launch_zero_words(void* p, uint64_t words, cudaStream_t st);
 // frame_bytes in sc.aux2[k] -> frame table, frame starts in sc.aux[k], header, *out_size
 cudaError_t launch_finalize(uint8_t* out, int codec, int dtype, uint64_t n, uint64_t F, uint32_t param,
                             const Scratch& sc, uint64_t* out_size, cudaStream_t st);
@@ -29,6 +31,7 @@ cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, c
 
 // zvc.cu
 uint32_t zvc_tiles(uint64_t n, int w, uint64_t F, uint32_t k0, uint32_t k1, uint32_t* tpf_out);
+void zvc_compress_scratch(uint64_t n, int w, uint64_t F, uint64_t* tiles, uint64_t* aux);
 cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
                                 const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st);
 cudaError_t launch_zvc_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,

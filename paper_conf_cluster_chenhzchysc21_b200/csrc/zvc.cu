@@ -65,7 +65,6 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar)))
                : "memory");
 }
-__device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, 256;" ::: "memory"); }
 
 // Read EPV elements starting at tile-relative element e0: from the smem stage where the bulk copy
 // landed, from global memory for the sub-16-byte tail of the tensor, zero past the tile end.
@@ -99,19 +98,33 @@ __device__ __forceinline__ uint4 tile_vec(const uint8_t* stage, const T* gsrc, u
 //                     stage                                                    (bar_empty[s])
 //   The consumers run (a)(b) of tile i+1 before (c) of tile i, so the offset latency overlaps.
 // ------------------------------------------------------------------------------------------
-constexpr int kProducerWarp = kWarps;
-// one resolver warp per stage: a resolver only ever waits on its own stage's barriers, so it can
-// never observe another phase's parity
-template <int S>
-constexpr int compress_threads() { return 32 * (kProducerWarp + 1 + S); }
+// warps [0, CW) consumers, warp CW producer, warps CW+1 .. CW+S resolvers: one resolver warp per
+// stage, so a resolver only ever waits on its own stage's barriers and can never observe another
+// phase's parity
+template <int S, int CW>
+constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 
-template <typename T, int S>
+#ifndef CSWAP_ZVC_DYNAMIC_TILES
+constexpr bool kStaticTiles = true;
+#else
+constexpr bool kStaticTiles = false;
+#endif
+
+// compress tile geometry: TB bytes per tile
+template <typename T, int TB>
+struct CGeom {
+  static constexpr int W = sizeof(T);
+  static constexpr int TILE = TB / W;  // elements per tile
+  static constexpr int WT = TILE / 32;  // bitmap words per tile
+};
+
+template <typename T, int S, int TB>
 struct CompressSmem {
-  using G = ZvcGeom<T>;
+  using G = CGeom<T, TB>;
   static constexpr uint32_t in_off = 0;
-  static constexpr uint32_t bm_off = S * kTileBytes + 128;  // +pad: shifted reads run <= 16 B past a stage
-  static constexpr uint32_t bytes = bm_off + S * G::WT * 4;
-  static constexpr int ctas_per_sm = bytes <= 110 * 1024 ? 2 : 1;
+  static constexpr uint32_t bytes = S * TB + 128;  // dynamic: the stage ring (+ pad)
+  static constexpr uint32_t static_bytes = S * G::WT * 4 + 1024;  // bitmap words, barriers, ...
+  static constexpr int ctas_per_sm = bytes + static_bytes <= 112 * 1024 ? 2 : 1;
 };
 
 __device__ __forceinline__ uint32_t spread16(uint32_t x) {  // bit i -> bit 2i (i < 16)
@@ -123,31 +136,38 @@ __device__ __forceinline__ uint32_t spread16(uint32_t x) {  // bit i -> bit 2i (
   return x;
 }
 
-template <typename T, int S>
-__global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::ctas_per_sm)
+// S stages; CW consumer warps; the consumers count tile i and emit tile i - LAG (LAG = S - 2),
+// so a tile's offset has LAG count phases of slack to resolve.
+template <typename T, int S, int CW, int TB>
+__global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, TB>::ctas_per_sm)
     zvc_compress_persistent(const T* __restrict__ in, uint64_t n, uint64_t F, uint32_t K, uint32_t tpf,
                             uint32_t num_tiles, uint8_t* __restrict__ out, uint64_t* out_size, Scratch sc,
                             uint32_t epoch, int dtype, int prof) {
   const uint32_t gpf = (tpf + 31) / 32;  // 32-tile groups per frame
-  using G = ZvcGeom<T>;
-  using L = CompressSmem<T, S>;
+  using G = CGeom<T, TB>;
+  using L = CompressSmem<T, S, TB>;
   constexpr uint32_t SENT = 0xFFFFFFFFu;
-  constexpr int ROWS = 32;                         // 4-byte loads per lane per tile
-  constexpr int WPR = sizeof(T) == 4 ? 1 : 2;      // bitmap words per row of 32 lanes
+  constexpr int kProducerWarp = CW;
+  constexpr int LAG = S - 2;
+  constexpr int PW = G::TILE / CW;   // elements per consumer warp (slab) per tile
+  constexpr int WPW = G::WT / CW;    // bitmap words per slab
+  static_assert(LAG >= 1 && PW % 256 == 0, "compress geometry");
   extern __shared__ __align__(128) uint8_t smem[];
   uint8_t* s_in = smem + L::in_off;
-  uint32_t* s_bm = reinterpret_cast<uint32_t*>(smem + L::bm_off);  // [S][WT] bitmap words per stage
+  // [S][WT] bitmap words per stage: a separate (static) array, so the compiler knows the
+  // bitmap stores never alias the stage loads and can batch the loads of a slab
+  __shared__ __align__(16) uint32_t s_bm[S * G::WT];
   __shared__ __align__(8) uint64_t bar_full[S], bar_empty[S], bar_cnt[S], bar_off[S];
   __shared__ uint32_t s_ticket[S];
   __shared__ uint32_t s_nnz[S];
-  __shared__ uint32_t s_wtot[S][kWarps];  // non-zeros per 1024-element slab, per stage
+  __shared__ uint32_t s_wtot[S][CW];  // non-zeros per slab, per stage
   __shared__ uint64_t s_off[S], s_fs[S];
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) {
     for (int s = 0; s < S; s++) {
       mbar_init(&bar_full[s], 1);
-      mbar_init(&bar_empty[s], kWarps);
+      mbar_init(&bar_empty[s], CW);
       mbar_init(&bar_cnt[s], 1);
       mbar_init(&bar_off[s], 1);
     }
@@ -169,9 +189,12 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
       long long c0 = clock64();
       if (i >= S) mbar_wait(&bar_empty[s], ((i / S) - 1) & 1);
       if (lane == 0) ZPROF_ADD(0, clock64() - c0);
-      uint32_t t = 0;
-      if (lane == 0) t = atomicAdd(sc.tickets + epoch, 1u);
-      t = __shfl_sync(0xffffffffu, t, 0);
+      // static round-robin assignment: CTA b takes tiles b, b + G, b + 2G, ... so every CTA
+      // counts the tiles of round r at about the same time and a tile's offset waits only for
+      // the skew between CTAs (a dynamic ticket would be claimed up to S-1 tiles before it is
+      // counted, and later tiles would wait for that prefetch lag)
+      const uint32_t t = kStaticTiles ? blockIdx.x + i * gridDim.x
+                                      : __shfl_sync(0xffffffffu, lane == 0 ? atomicAdd(sc.tickets + epoch, 1u) : 0u, 0);
       if (t >= num_tiles) {
         if (lane == 0) {
           s_ticket[s] = SENT;
@@ -186,7 +209,7 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
         s_ticket[s] = t;
         if (be) {
           mbar_expect_tx(&bar_full[s], be * G::W);
-          bulk_g2s(s_in + s * kTileBytes, in + uint64_t(k) * F + uint64_t(j) * G::TILE, be * G::W, &bar_full[s]);
+          bulk_g2s(s_in + s * TB, in + uint64_t(k) * F + uint64_t(j) * G::TILE, be * G::W, &bar_full[s]);
         } else {
           mbar_arrive(&bar_full[s]);
         }
@@ -288,22 +311,22 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
   }
 
   // ------------------------------------------------------------------------- consumers
-  // 8 warps, warp w owns slab w (1024 elements = 32 rows of 32 four-byte words) of every tile.
+  // CW warps, warp w owns slab w (PW elements = PW/32 rows of 32 words) of every tile.
   // count(i):   rows -> one ballot per row = one bitmap word (fp32) / two ballots (16-bit);
   //             slab totals; the tile count is published (A) and added to the accumulators.
   // emit(i-1):  wait for tile i-1's offset, re-read its rows from the stage and store every
   //             non-zero straight to global memory at its rank (a warp's predicated 4-byte
   //             stores of one row cover a contiguous range); store the slab's bitmap words.
-  // count(i) runs before emit(i-1), so a tile's count never waits for an older tile's offset.
+  // count(i) runs before emit(i-LAG), so a tile's count never waits for an older tile's offset.
   const uint32_t lt = (1u << lane) - 1u;
-  constexpr uint32_t SLAB = G::PER_WARP * G::W;  // bytes per slab (4 KiB)
+  auto consumer_sync = [] { asm volatile("bar.sync 1, %0;" ::"n"(32 * CW) : "memory"); };
   // element e of the tile: from the stage (bulk-copied part), the global tail, or zero
   auto load_elem = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t e, uint32_t te, uint32_t be) {
     constexpr bool full = decltype(full_tag)::value;
     if (full) return uint32_t(reinterpret_cast<const T*>(stage)[e]);
     return e < be ? uint32_t(reinterpret_cast<const T*>(stage)[e]) : (e < te ? uint32_t(gsrc[e]) : 0u);
   };
-  constexpr int EROWS = G::PER_WARP / 32;  // rows of 32 elements per slab (32 fp32 / 64 fp16)
+  constexpr int EROWS = PW / 32;  // rows of 32 elements per slab
   auto group_wait = [&](uint64_t* bar, uint32_t parity) {  // one warp polls, the rest block in bar.sync
     if (warp == 0) mbar_wait(bar, parity);
     consumer_sync();
@@ -313,20 +336,28 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
   auto count_slab = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be,
                         uint32_t* bm_out) {
     // row m = elements [32m, 32m+32) of the slab: one ballot is bitmap word (slab word m)
-    const uint32_t e0 = warp * G::PER_WARP + lane;
+    // rows in batches of 16: the batch's loads are issued before its ballots and bitmap stores
+    // (the compiler does not move shared loads across a ballot followed by a shared store)
+    constexpr int B = EROWS < 16 ? EROWS : 16;
+    const uint32_t e0 = warp * PW + lane;
     uint32_t tot = 0;
-#pragma unroll 8
-    for (int m = 0; m < EROWS; m++) {
-      const uint32_t v = load_elem(full_tag, stage, gsrc, e0 + 32 * m, te, be);
-      const uint32_t w = __ballot_sync(0xffffffffu, v != 0);
-      if (lane == 0) bm_out[m] = w;
-      tot += __popc(w);
+#pragma unroll
+    for (int m0 = 0; m0 < EROWS; m0 += B) {
+      uint32_t v[B];
+#pragma unroll
+      for (int u = 0; u < B; u++) v[u] = load_elem(full_tag, stage, gsrc, e0 + 32 * (m0 + u), te, be);
+#pragma unroll
+      for (int u = 0; u < B; u++) {
+        const uint32_t w = __ballot_sync(0xffffffffu, v[u] != 0);
+        if (lane == 0) bm_out[m0 + u] = w;
+        tot += __popc(w);
+      }
     }
     return tot;
   };
 
   auto emit_slab = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be, uint8_t* dst) {
-    const uint32_t e0 = warp * G::PER_WARP + lane;
+    const uint32_t e0 = warp * PW + lane;
     uint32_t pre = 0;
 #pragma unroll 8
     for (int m = 0; m < EROWS; m++) {
@@ -343,8 +374,8 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
     uint64_t Fk;
     tile_geom(t, k, j, Fk, te, be);
     const T* gsrc = in + uint64_t(k) * F + uint64_t(j) * G::TILE;
-    const uint8_t* stage = s_in + s * kTileBytes;
-    uint32_t* bm_out = s_bm + s * G::WT + warp * (G::WT / kWarps);
+    const uint8_t* stage = s_in + s * TB;
+    uint32_t* bm_out = s_bm + s * G::WT + warp * WPW;
     const uint32_t c = (te == G::TILE && be == G::TILE) ? count_slab(std::true_type{}, stage, gsrc, te, be, bm_out)
                                                         : count_slab(std::false_type{}, stage, gsrc, te, be, bm_out);
     if (lane == 0) s_wtot[s][warp] = c;
@@ -352,7 +383,7 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
     if (tid == 0) {  // publish the tile count (A) and feed the frame / group accumulators
       uint32_t tot = 0;
 #pragma unroll
-      for (int w = 0; w < kWarps; w++) tot += s_wtot[s][w];
+      for (int w = 0; w < CW; w++) tot += s_wtot[s][w];
       st_relaxed(sc.status + t, make_status(tot, epoch, kFlagA));  // self-contained: no release needed
       atomicAdd(reinterpret_cast<unsigned long long*>(sc.aux2 + k), (1ull << 40) + tot);
       atomicAdd(reinterpret_cast<unsigned long long*>(sc.aux2 + K + uint64_t(k) * gpf + j / 32), (1ull << 40) + tot);
@@ -372,10 +403,10 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
     uint64_t Fk;
     tile_geom(t, k, j, Fk, te, be);
     const T* gsrc = in + uint64_t(k) * F + uint64_t(j) * G::TILE;
-    const uint8_t* stage = s_in + s * kTileBytes;
+    const uint8_t* stage = s_in + s * TB;
     uint32_t woff = 0, nnz = 0;
 #pragma unroll
-    for (int w = 0; w < kWarps; w++) {
+    for (int w = 0; w < CW; w++) {
       const uint32_t x = s_wtot[s][w];
       woff += w < warp ? x : 0;
       nnz += x;
@@ -384,7 +415,6 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
     if (te == G::TILE && be == G::TILE) emit_slab(std::true_type{}, stage, gsrc, te, be, dst);
     else emit_slab(std::false_type{}, stage, gsrc, te, be, dst);
     {  // this slab's bitmap words, clipped to the frame's bitmap section (incl. its 16-byte pad)
-      constexpr uint32_t WPW = G::WT / kWarps;
       const uint64_t wsec = (cdiv(Fk, 32) + 3) & ~uint64_t(3);
       const uint64_t w0 = uint64_t(j) * G::WT + warp * WPW;
       if (w0 < wsec) {
@@ -397,7 +427,7 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
     __syncwarp();
     if (lane == 0) mbar_arrive(&bar_empty[s]);  // this warp no longer reads the stage
     const uint64_t g1 = g0 + uint64_t(nnz) * G::W;
-    if (warp == kWarps - 1 && lane == 31) {
+    if (warp == CW - 1 && lane == 31) {
       if (uint64_t(j) * G::TILE + G::TILE >= Fk) {  // last tile of the frame: pad + frame_bytes[k]
         for (uint64_t b = g1; b < a16(g1); b += 2) *reinterpret_cast<uint16_t*>(out + b) = 0;
         *reinterpret_cast<uint64_t*>(out + 64 + 8ull * k) = a16(g1) - fstart;
@@ -412,7 +442,7 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
     if (tid == 0) ZPROF_ADD(6, clock64() - c2);
   };
 
-  uint32_t prev_t = SENT;
+  // a pending tile's ticket stays in s_ticket[its stage] until its emit releases the stage
   for (uint32_t i = 0;; i++) {
     const int s = i % S;
     long long c0 = clock64();
@@ -420,20 +450,20 @@ __global__ void __launch_bounds__(compress_threads<S>(), CompressSmem<T, S>::cta
     if (tid == 0) ZPROF_ADD(7, clock64() - c0);
     const uint32_t t = s_ticket[s];
     if (t == SENT) {
-      if (tid == 0) {  // no more work: tell every resolver
+      for (uint32_t p = i > uint32_t(LAG) ? i - LAG : 0; p < i; p++) emit(p, s_ticket[p % S]);
+      // every pending tile is resolved (its resolver has read s_nnz): now stop the resolvers
+      if (tid == 0) {
         for (uint32_t i2 = i; i2 < i + S; i2++) {
           s_nnz[i2 % S] = SENT;
           mbar_arrive(&bar_cnt[i2 % S]);
         }
       }
-      if (prev_t != SENT) emit(i - 1, prev_t);
       break;
     }
     long long c3 = clock64();
     count(i, t);
     if (tid == 0) ZPROF_ADD(8, clock64() - c3);
-    if (prev_t != SENT) emit(i - 1, prev_t);
-    prev_t = t;
+    if (i >= uint32_t(LAG)) emit(i - LAG, s_ticket[(i - LAG) % S]);
   }
 }
 
@@ -649,34 +679,35 @@ static int sm_count() {
   return sms;
 }
 
-template <typename T, int S>
+template <typename T, int S, int CW, int TB>
 static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uint8_t* out, uint64_t* out_size,
                                      const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st) {
-  using L = CompressSmem<T, S>;
+  using L = CompressSmem<T, S, TB>;
   const uint32_t K = uint32_t(cdiv(n, F));
-  uint32_t tpf;
-  const uint32_t tiles = zvc_tiles(n, sizeof(T), F, 0, K, &tpf);
+  const uint32_t TILE = TB / sizeof(T);
+  const uint32_t tpf = uint32_t(cdiv(F, TILE));
+  const uint32_t tiles = (K - 1) * tpf + uint32_t(cdiv(frame_len(n, F, K - 1), TILE));
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(zvc_compress_persistent<T, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, L::bytes);
+    cudaFuncSetAttribute(zvc_compress_persistent<T, S, CW, TB>, cudaFuncAttributeMaxDynamicSharedMemorySize, L::bytes);
     attr = true;
   }
   const uint32_t per_sm = L::ctas_per_sm;
   // per-frame and per-group (tiles, nnz) accumulators
-  cudaMemsetAsync(sc.aux2, 0, (uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32)) * 8, st);
+  launch_zero_words(sc.aux2, (uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32)) * 2, st);
   const uint32_t grid = std::min<uint32_t>(tiles, uint32_t(sm_count()) * per_sm);
   timing_kernel_start(st);
-  zvc_compress_persistent<T, S><<<grid, compress_threads<S>(), L::bytes, st>>>(
+  zvc_compress_persistent<T, S, CW, TB><<<grid, compress_threads<S, CW>(), L::bytes, st>>>(
       static_cast<const T*>(in), n, F, K, tpf, tiles, out, out_size, sc, epoch, dtype, prof_enabled());
   if (prof_enabled()) {
     unsigned long long h[16];
     cudaStreamSynchronize(st);
     cudaMemcpyFromSymbol(h, g_zprof, sizeof(h));
     fprintf(stderr,
-            "[zprof] grid=%u tiles=%u | per-tile cycles: producer_wait_empty=%.0f counter_wait_full=%.0f "
+            "[zprof] TB=%d S=%d CW=%d grid=%u tiles=%u | per-tile cycles: producer_wait_empty=%.0f "
             "resolver_wait_cnt=%.0f resolver_lookback=%.0f | consumer(tid0): wait_off=%.0f finish=%.0f "
             "wait_full=%.0f prep=%.0f\n",
-            grid, tiles, h[0] / double(tiles), h[1] / double(tiles), h[2] / double(tiles), h[3] / double(tiles),
+            TB, S, CW, grid, tiles, h[0] / double(tiles), h[2] / double(tiles), h[3] / double(tiles),
             h[5] / double(tiles), h[6] / double(tiles), h[7] / double(tiles), h[8] / double(tiles));
     memset(h, 0, sizeof(h));
     cudaMemcpyToSymbol(g_zprof, h, sizeof(h));
@@ -684,25 +715,34 @@ static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uin
   return cudaGetLastError();
 }
 
-static int stages_cfg() {
-  static int s = -1;
-  if (s < 0) {
-    const char* e = getenv("CSWAP_ZVC_STAGES");
-    s = e ? atoi(e) : 3;
-    if (s < 2 || s > 6) s = 3;
+// compress configuration (stages x consumer warps); CSWAP_ZVC_CFG overrides for experiments
+static int compress_cfg() {
+  static int c = -1;
+  if (c < 0) {
+    const char* e = getenv("CSWAP_ZVC_CFG");
+    c = e ? atoi(e) : 0;
+    if (c < 0 || c > 3) c = 0;
   }
-  return s;
+  return c;
 }
 
 template <typename T>
 static cudaError_t launch_compress_t(const void* in, uint64_t n, uint64_t F, uint8_t* out, uint64_t* out_size,
                                      const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st) {
-  switch (stages_cfg()) {
-    case 2: return launch_compress_s<T, 2>(in, n, F, out, out_size, sc, epoch, dtype, st);
-    case 4: return launch_compress_s<T, 4>(in, n, F, out, out_size, sc, epoch, dtype, st);
-    case 5: return launch_compress_s<T, 5>(in, n, F, out, out_size, sc, epoch, dtype, st);
-    default: return launch_compress_s<T, 3>(in, n, F, out, out_size, sc, epoch, dtype, st);
+  switch (compress_cfg()) {
+    case 1: return launch_compress_s<T, 6, 8, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    case 2: return launch_compress_s<T, 5, 8, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    case 3: return launch_compress_s<T, 4, 8, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    default: return launch_compress_s<T, 3, 8, 32768>(in, n, F, out, out_size, sc, epoch, dtype, st);
   }
+}
+
+// scratch a compress launch needs: tile status words and (frame + 32-tile group) accumulators,
+// sized for the smallest compress tile any configuration uses (16 KiB)
+void zvc_compress_scratch(uint64_t n, int w, uint64_t F, uint64_t* tiles, uint64_t* aux) {
+  const uint64_t TILE = 16384 / w, K = cdiv(n, F), tpf = cdiv(F, TILE);
+  *tiles = K ? (K - 1) * tpf + cdiv(frame_len(n, F, K - 1), TILE) : 0;
+  *aux = K + K * ((tpf + 31) / 32) + 2;
 }
 
 cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
