@@ -104,6 +104,12 @@ __device__ __forceinline__ uint4 tile_vec(const uint8_t* stage, const T* gsrc, u
 template <int S, int CW>
 constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 
+// resolver polling: __nanosleep backoff bounds (ns)
+#ifndef CSWAP_ZVC_MAX_BACKOFF
+#define CSWAP_ZVC_MAX_BACKOFF 32
+#endif
+constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
+
 #ifndef CSWAP_ZVC_DYNAMIC_TILES
 constexpr bool kStaticTiles = true;
 #else
@@ -240,17 +246,17 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           fstart = data_start(K);
         } else {  // previous frame's start + its bitmap + its packed values (from its accumulator)
           uint64_t a, acc;
-          uint32_t backoff = 32;
+          uint32_t backoff = kMinBackoff;
           while (status_flag(a = ld_relaxed(sc.aux + k - 1), epoch) != kFlagP) {
             __nanosleep(backoff);
-            backoff = backoff < 256 ? backoff * 2 : 256;
+            backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
           }
           const uint64_t Fp = frame_len(n, F, k - 1);
           const uint64_t tiles_prev = cdiv(Fp, G::TILE);
           backoff = 32;
           while (((acc = ld_relaxed(sc.aux2 + k - 1)) >> 40) != tiles_prev) {
             __nanosleep(backoff);
-            backoff = backoff < 256 ? backoff * 2 : 256;
+            backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
           }
           fstart = status_value(a) + a16(4 * cdiv(Fp, 32)) + a16(G::W * (acc & ((1ull << 40) - 1)));
         }
@@ -264,10 +270,10 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           uint64_t v = 0;
           if (gi < g) {
             const uint64_t* p = sc.aux2 + K + uint64_t(k) * gpf + gi;
-            uint32_t backoff = 32;
+            uint32_t backoff = kMinBackoff;
             while (((v = ld_relaxed(p)) >> 40) != 32) {
               __nanosleep(backoff);
-              backoff = backoff < 256 ? backoff * 2 : 256;
+              backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
             }
             v &= (1ull << 40) - 1;
           }
@@ -278,10 +284,10 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         if (uint32_t(lane) < jj) {
           const uint64_t* p = sc.status + (t - jj + lane);
           uint64_t st;
-          uint32_t backoff = 32;
+          uint32_t backoff = kMinBackoff;
           while (status_flag(st = ld_relaxed(p), epoch) == 0) {
             __nanosleep(backoff);
-            backoff = backoff < 256 ? backoff * 2 : 256;
+            backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
           }
           v = status_value(st);
         }
@@ -290,10 +296,10 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       if (lane == 0) {
         if (j != 0) {
           uint64_t a;
-          uint32_t backoff = 32;
+          uint32_t backoff = kMinBackoff;
           while (status_flag(a = ld_relaxed(sc.aux + k), epoch) != kFlagP) {
             __nanosleep(backoff);
-            backoff = backoff < 256 ? backoff * 2 : 256;
+            backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
           }
           fstart = status_value(a);
         }
@@ -333,13 +339,15 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     if (warp != 0) mbar_wait(bar, parity);  // phase already complete: returns at once
   };
 
-  auto count_slab = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be,
+  auto count_slab = [&](auto full_tag, uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be,
                         uint32_t* bm_out) {
-    // row m = elements [32m, 32m+32) of the slab: one ballot is bitmap word (slab word m)
-    // rows in batches of 16: the batch's loads are issued before its ballots and bitmap stores
-    // (the compiler does not move shared loads across a ballot followed by a shared store)
+    // row m = elements [32m, 32m+32) of the slab: one ballot is bitmap word (slab word m); the
+    // non-zeros are compacted in place to the start of the slab (a row's writes land at or
+    // before the row, and every row of a batch is loaded before any of its writes).
+    // Rows go in batches of 16 so the batch's loads issue back to back.
     constexpr int B = EROWS < 16 ? EROWS : 16;
     const uint32_t e0 = warp * PW + lane;
+    T* sv = reinterpret_cast<T*>(stage) + warp * PW;
     uint32_t tot = 0;
 #pragma unroll
     for (int m0 = 0; m0 < EROWS; m0 += B) {
@@ -350,22 +358,21 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       for (int u = 0; u < B; u++) {
         const uint32_t w = __ballot_sync(0xffffffffu, v[u] != 0);
         if (lane == 0) bm_out[m0 + u] = w;
+        if (v[u]) sv[tot + __popc(w & lt)] = T(v[u]);
         tot += __popc(w);
       }
     }
+    __syncwarp();
     return tot;
   };
 
-  auto emit_slab = [&](auto full_tag, const uint8_t* stage, const T* gsrc, uint32_t te, uint32_t be, uint8_t* dst) {
-    const uint32_t e0 = warp * PW + lane;
-    uint32_t pre = 0;
-#pragma unroll 8
-    for (int m = 0; m < EROWS; m++) {
-      const uint32_t v = load_elem(full_tag, stage, gsrc, e0 + 32 * m, te, be);
-      const uint32_t w = __ballot_sync(0xffffffffu, v != 0);
-      if (v) reinterpret_cast<T*>(dst)[pre + __popc(w & lt)] = T(v);
-      pre += __popc(w);
-    }
+  // copy the slab's compacted non-zeros (count_slab) to the container: full-warp stores of
+  // consecutive words
+  auto emit_slab = [&](const uint8_t* stage, uint32_t cnt, uint8_t* dst) {
+    const T* sv = reinterpret_cast<const T*>(stage) + warp * PW;
+    T* d = reinterpret_cast<T*>(dst);
+#pragma unroll 4
+    for (uint32_t q = lane; q < cnt; q += 32) d[q] = sv[q];
   };
 
   auto count = [&](uint32_t i, uint32_t t) {
@@ -374,7 +381,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     uint64_t Fk;
     tile_geom(t, k, j, Fk, te, be);
     const T* gsrc = in + uint64_t(k) * F + uint64_t(j) * G::TILE;
-    const uint8_t* stage = s_in + s * TB;
+    uint8_t* stage = s_in + s * TB;
     uint32_t* bm_out = s_bm + s * G::WT + warp * WPW;
     const uint32_t c = (te == G::TILE && be == G::TILE) ? count_slab(std::true_type{}, stage, gsrc, te, be, bm_out)
                                                         : count_slab(std::false_type{}, stage, gsrc, te, be, bm_out);
@@ -402,7 +409,6 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     uint32_t k, j, te, be;
     uint64_t Fk;
     tile_geom(t, k, j, Fk, te, be);
-    const T* gsrc = in + uint64_t(k) * F + uint64_t(j) * G::TILE;
     const uint8_t* stage = s_in + s * TB;
     uint32_t woff = 0, nnz = 0;
 #pragma unroll
@@ -412,8 +418,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       nnz += x;
     }
     uint8_t* dst = out + g0 + uint64_t(G::W) * woff;
-    if (te == G::TILE && be == G::TILE) emit_slab(std::true_type{}, stage, gsrc, te, be, dst);
-    else emit_slab(std::false_type{}, stage, gsrc, te, be, dst);
+    emit_slab(stage, s_wtot[s][warp], dst);
     {  // this slab's bitmap words, clipped to the frame's bitmap section (incl. its 16-byte pad)
       const uint64_t wsec = (cdiv(Fk, 32) + 3) & ~uint64_t(3);
       const uint64_t w0 = uint64_t(j) * G::WT + warp * WPW;
