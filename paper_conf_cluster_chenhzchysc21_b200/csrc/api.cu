@@ -689,7 +689,8 @@ static cswap_status probe_impl(Ctx* c, const void* d_in, uint64_t n, int dtype, 
   uint64_t* counts = reinterpret_cast<uint64_t*>(slot);
   cudaEvent_t ev;
   cswap_status s = CSWAP_OK;
-  if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming | cudaEventBlockingSync) != cudaSuccess) {
+  // spin-wait event: a blocking-sync event sleeps in the OS and wakes ~100 us late
+  if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) {
     c->pinned.free(slot);
     return fail(CSWAP_ERR_CUDA, "event create failed");
   }

@@ -172,7 +172,10 @@ __global__ void __launch_bounds__(1024) prep_kernel(const uint8_t* in, uint64_t 
     if (!ok) set_error(err, kErrCorrupt);
   }
   __syncthreads();
-  if (!s_ok) return;
+  if (!s_ok) {
+    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) fstart[k] = fbytes[k] = 0;
+    return;
+  }
   const uint64_t* table = reinterpret_cast<const uint64_t*>(in + 64);
   const uint64_t base = data_start(K);
   uint64_t carry = 0;
@@ -189,8 +192,17 @@ __global__ void __launch_bounds__(1024) prep_kernel(const uint8_t* in, uint64_t 
     }
     carry += tot;
   }
-  if (bad) set_error(err, kErrCorrupt);
-  if (threadIdx.x == 0 && base + carry != s_total) set_error(err, kErrCorrupt);
+  // a bad frame table leaves every frame empty (start 0, 0 bytes): single-pass decoders, which
+  // cannot stop early without stalling their successors, then see a size mismatch and read nothing
+  __shared__ int s_bad;
+  if (threadIdx.x == 0) s_bad = 0;
+  __syncthreads();
+  if (bad || (threadIdx.x == 0 && base + carry != s_total)) s_bad = 1;
+  __syncthreads();
+  if (s_bad) {
+    if (threadIdx.x == 0) set_error(err, kErrCorrupt);
+    for (uint32_t k = threadIdx.x; k < K; k += blockDim.x) fstart[k] = fbytes[k] = 0;
+  }
 }
 
 cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
@@ -262,11 +274,12 @@ __global__ void __launch_bounds__(kThreads) probe_kernel(const T* __restrict__ x
   __syncthreads();
   if (threadIdx.x == 0) s_last = atomicAdd(done, 1u) == gridDim.x - 1;
   __syncthreads();
-  if (s_last && threadIdx.x < 3) {
+  if (s_last && warp < 3) {  // warp c sums counter c over the CTAs' partials
     __threadfence();
     uint64_t a = 0;
-    for (uint32_t b = 0; b < gridDim.x; b++) a += reinterpret_cast<volatile uint64_t*>(partial)[b * 3 + threadIdx.x];
-    counts3[threadIdx.x] = a;
+    for (uint32_t b = lane; b < gridDim.x; b += 32) a += __ldcg(partial + b * 3 + warp);
+    a = warp_sum_u64(a);
+    if (lane == 0) counts3[warp] = a;
   }
 }
 

@@ -758,7 +758,9 @@ cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, u
 
 template <typename T>
 static cudaError_t launch_zvc_decompress_t(const uint8_t* in, void* out, uint64_t n, uint64_t F, uint32_t k0,
-                                           uint32_t k1, const Scratch& sc, uint32_t* err, cudaStream_t st) {
+                                           uint32_t k1, const Scratch& sc, uint32_t epoch, uint32_t* err,
+                                           cudaStream_t st) {
+  (void)epoch;  // the split decode needs no inter-CTA status words
   uint32_t tpf;
   const uint32_t tiles = zvc_tiles(n, sizeof(T), F, k0, k1, &tpf);
   if (!tiles) return cudaSuccess;
@@ -776,9 +778,9 @@ static cudaError_t launch_zvc_decompress_t(const uint8_t* in, void* out, uint64_
 }
 
 cudaError_t launch_zvc_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
-                                  uint32_t k1, const Scratch& sc, uint32_t /*epoch*/, uint32_t* err, cudaStream_t st) {
-  return w == 4 ? launch_zvc_decompress_t<uint32_t>(in, out, n, F, k0, k1, sc, err, st)
-                : launch_zvc_decompress_t<uint16_t>(in, out, n, F, k0, k1, sc, err, st);
+                                  uint32_t k1, const Scratch& sc, uint32_t epoch, uint32_t* err, cudaStream_t st) {
+  return w == 4 ? launch_zvc_decompress_t<uint32_t>(in, out, n, F, k0, k1, sc, epoch, err, st)
+                : launch_zvc_decompress_t<uint16_t>(in, out, n, F, k0, k1, sc, epoch, err, st);
 }
 
 }  // namespace cswap
