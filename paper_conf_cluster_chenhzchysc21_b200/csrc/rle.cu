@@ -8,8 +8,8 @@
 // The values section starts after all r lengths, so a tile can only place its runs once the
 // whole frame is counted; compress is therefore: count (run starts per tile + first start) ->
 // per-frame scan (run offsets, next run start after each tile, r_k) -> frame table -> emit.
-// Decompress: per-frame scan of the lengths into run start positions, then one CTA per output
-// tile where every element finds its run by binary search.
+// Decompress: chunked scan of the lengths (chunk sums -> per-frame scan of the chunk sums), then
+// one CTA per output tile paints the runs overlapping it (see rle_paint_kernel).
 #include "kernels.h"
 #include "tile_common.cuh"
 
@@ -200,91 +200,183 @@ cudaError_t launch_rle_compress(const void* in, uint64_t n, int w, uint64_t F, u
 // decompress
 // ------------------------------------------------------------------------------------------
 // one CTA per frame: validate, run start positions (frame-relative) into rs[k*F + i]
-template <typename T>
-__global__ void __launch_bounds__(1024) rle_dscan_kernel(const uint8_t* __restrict__ in, uint64_t n, uint64_t F,
-                                                         uint32_t k0, uint32_t* rs, Scratch sc, uint32_t* err) {
-  using G = TileGeom<T>;
+// ---- decompress ------------------------------------------------------------------------------
+// The lengths of frame k are cut into chunks of kRleChunk runs.  (1) one CTA per chunk slot sums
+// its chunk's lengths; (2) one CTA per frame validates the frame and scans the chunk sums into
+// chunk start positions; (3) one CTA per output tile finds the chunk holding its first element
+// (32-ary search over the frame's chunk starts), then for each chunk overlapping the tile scans
+// the chunk's lengths in shared memory into run starts and paints every run's clipped range
+// into a shared-memory copy of the tile (short runs by one thread, runs longer than 32 elements
+// by a whole warp), and stores the tile with 16-byte stores.  Traffic: lengths twice (the
+// second read mostly from L2), values once, output once.
+constexpr uint32_t kRleChunk = 1024;
+
+__device__ __forceinline__ bool rle_frame_header(const uint8_t* in, uint64_t fstart, uint64_t fb, uint64_t Fk, int w,
+                                                 uint64_t* r_out) {
+  if (fb < 16) return false;
+  const uint64_t r = *reinterpret_cast<const uint32_t*>(in + fstart);
+  *r_out = r;
+  return r >= 1 && r <= Fk && fb == 16 + a16(4 * r) + a16(uint64_t(w) * r);
+}
+
+// one warp per chunk slot, grid-stride (most slots of a frame are empty when runs are long)
+__global__ void __launch_bounds__(kThreads) rle_dsum_kernel(const uint8_t* __restrict__ in, uint64_t n, uint64_t F,
+                                                            int w, uint32_t k0, uint32_t k1, uint32_t cpf,
+                                                            uint64_t* csum, Scratch sc, uint32_t* err) {
+  if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
+  const int lane = threadIdx.x & 31;
+  const uint64_t slots = uint64_t(k1 - k0) * cpf;
+  const uint64_t nwarps = uint64_t(gridDim.x) * kWarps;
+  for (uint64_t sl = uint64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); sl < slots; sl += nwarps) {
+    const uint32_t k = k0 + uint32_t(sl / cpf), c = uint32_t(sl % cpf);
+    const uint64_t Fk = frame_len(n, F, k);
+    uint64_t r;
+    if (!rle_frame_header(in, sc.aux[k], sc.aux2[k], Fk, w, &r)) continue;  // flagged by rle_dscan2
+    const uint64_t i0 = uint64_t(c) * kRleChunk;
+    if (i0 >= r) {  // past the frame's last chunk: skip the rest of this frame's slots
+      continue;
+    }
+    const uint32_t m = uint32_t(umin64(kRleChunk, r - i0));
+    const uint32_t* len = reinterpret_cast<const uint32_t*>(in + sc.aux[k] + 16) + i0;
+    uint64_t acc = 0;  // <= kRleChunk * 2^32
+    bool zero = false;
+#pragma unroll 8
+    for (uint32_t i = lane; i < m; i += 32) {
+      const uint32_t v = len[i];
+      zero |= v == 0;
+      acc += v;
+    }
+    if (__any_sync(0xffffffffu, zero) && lane == 0) set_error(err, kErrCorrupt);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (lane == 0) csum[sl] = acc;
+  }
+}
+
+__global__ void __launch_bounds__(1024) rle_dscan2_kernel(const uint8_t* __restrict__ in, uint64_t n, uint64_t F,
+                                                          int w, uint32_t k0, uint32_t cpf, uint64_t* csum,
+                                                          Scratch sc, uint32_t* err) {
   __shared__ uint64_t s_tmp[33];
   __shared__ int s_ok;
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const uint32_t k = k0 + blockIdx.x;
   const uint64_t Fk = frame_len(n, F, k);
-  const uint64_t fstart = sc.aux[k], fb = sc.aux2[k];
   if (threadIdx.x == 0) {
-    int ok = fb >= 16;
-    uint64_t r = ok ? *reinterpret_cast<const uint32_t*>(in + fstart) : 0;
-    ok = ok && r >= 1 && r <= Fk && fb == 16 + a16(4 * r) + a16(uint64_t(G::W) * r);
+    uint64_t r = 0;
+    const bool ok = rle_frame_header(in, sc.aux[k], sc.aux2[k], Fk, w, &r);
     sc.aux3[k] = ok ? r : 0;
     s_ok = ok;
     if (!ok) set_error(err, kErrCorrupt);
   }
   __syncthreads();
   if (!s_ok) return;
-  const uint64_t r = sc.aux3[k];
-  const uint32_t* len = reinterpret_cast<const uint32_t*>(in + fstart + 16);
-  uint32_t* out = rs + uint64_t(k) * F;
+  const uint32_t nch = uint32_t(cdiv(sc.aux3[k], kRleChunk));
+  uint64_t* cs = csum + uint64_t(blockIdx.x) * cpf;
   uint64_t carry = 0;
-  bool bad = false;
-  for (uint64_t c0 = 0; c0 < r; c0 += blockDim.x) {
-    const uint64_t i = c0 + threadIdx.x;
-    const uint64_t v = i < r ? len[i] : 0;
-    bad |= i < r && v == 0;
+  for (uint32_t c0 = 0; c0 < nch; c0 += blockDim.x) {
+    const uint32_t c = c0 + threadIdx.x;
+    const uint64_t v = c < nch ? cs[c] : 0;
     uint64_t tot;
     const uint64_t ex = block_excl_sum_u64(v, s_tmp, &tot);
-    if (i < r) out[i] = uint32_t(umin64(carry + ex, Fk));
+    if (c < nch) cs[c] = carry + ex;  // chunk start position inside the frame
     carry += tot;
   }
-  if (bad || carry != Fk) set_error(err, kErrCorrupt);
+  if (threadIdx.x == 0 && carry != Fk) set_error(err, kErrCorrupt);
 }
 
-// one CTA per output tile: element e -> run = last start <= e (binary search), value of that run
 template <typename T>
-__global__ void __launch_bounds__(kThreads) rle_expand_kernel(const uint8_t* __restrict__ in, T* __restrict__ outp,
-                                                              uint64_t n, uint64_t F, uint32_t tpf, uint32_t k0,
-                                                              const uint32_t* rs, Scratch sc, uint32_t* err) {
+__global__ void __launch_bounds__(kThreads) rle_paint_kernel(const uint8_t* __restrict__ in, T* __restrict__ outp,
+                                                             uint64_t n, uint64_t F, uint32_t tpf, uint32_t k0,
+                                                             uint32_t cpf, const uint64_t* __restrict__ cstart,
+                                                             Scratch sc, uint32_t* err) {
   using G = TileGeom<T>;
-  __shared__ uint64_t s_lo, s_hi;
+  __shared__ __align__(16) T s_out[G::TILE];
+  __shared__ uint32_t s_len[kRleChunk];
+  __shared__ T s_val[kRleChunk];
+  __shared__ uint64_t s_tmp[33];
+  __shared__ uint32_t s_long[G::TILE / 33 + 2][3];  // runs longer than 32 elements inside the tile: (a, b, value)
+  __shared__ uint32_t s_nlong, s_c0;
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const uint32_t t = blockIdx.x + k0 * tpf;
   const TilePos p = tile_pos<T>(t, n, F, tpf);
   const uint64_t r = sc.aux3[p.k];
   if (r == 0) return;
-  const uint32_t* st = rs + uint64_t(p.k) * F;
-  const T* values = reinterpret_cast<const T*>(in + sc.aux[p.k] + 16 + a16(4 * r));
+  const uint32_t nch = uint32_t(cdiv(r, kRleChunk));
+  const uint64_t* cs = cstart + uint64_t(p.k - k0) * cpf;
+  const uint32_t* lens = reinterpret_cast<const uint32_t*>(in + sc.aux[p.k] + 16);
+  const T* vals = reinterpret_cast<const T*>(in + sc.aux[p.k] + 16 + a16(4 * r));
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  // warps 0/1: 32-ary search for the runs holding the tile's first / last element
-  if (warp < 2) {
-    const uint64_t target = warp == 0 ? p.tin : p.tin + p.te - 1;
-    uint64_t lo = 0, hi = r;  // answer in [lo, hi): last i with st[i] <= target
+  const uint64_t tb = p.tin, te = p.tin + p.te;
+  if (warp == 0) {  // last chunk with start <= tb (chunk 0 starts at 0)
+    uint32_t lo = 0, hi = nch;
     while (hi - lo > 1) {
-      const uint64_t span = hi - lo;
-      const uint64_t probe = lo + (span * uint64_t(lane)) / 32;
-      const bool le = st[probe] <= target;
-      const uint32_t m = __ballot_sync(0xffffffffu, le);
-      const int last = 31 - __clz(m);  // lane 0 always satisfies (st[lo] <= target)
-      const uint64_t nlo = lo + (span * uint64_t(last)) / 32;
-      const uint64_t nhi = last == 31 ? hi : lo + (span * uint64_t(last + 1)) / 32;
+      const uint32_t span = hi - lo;
+      const uint32_t probe = lo + uint32_t((uint64_t(span) * lane) / 32);
+      const uint32_t m = __ballot_sync(0xffffffffu, cs[probe] <= tb);
+      const int last = 31 - __clz(m);
+      const uint32_t nlo = lo + uint32_t((uint64_t(span) * last) / 32);
+      const uint32_t nhi = last == 31 ? hi : lo + uint32_t((uint64_t(span) * (last + 1)) / 32);
       lo = nlo;
       hi = nhi > nlo ? nhi : nlo + 1;
     }
-    if (lane == 0) {
-      if (warp == 0) s_lo = lo;
-      else s_hi = lo;
-    }
+    if (lane == 0) s_c0 = lo;
   }
   __syncthreads();
-  const uint64_t rlo = s_lo, rhi = s_hi;
-  T* dst = outp + uint64_t(p.k) * F + p.tin;
-  for (uint32_t e = threadIdx.x; e < p.te; e += blockDim.x) {
-    const uint64_t pos = p.tin + e;
-    uint64_t lo = rlo, hi = rhi + 1;
-    while (hi - lo > 1) {
-      const uint64_t mid = (lo + hi) / 2;
-      if (st[mid] <= pos) lo = mid;
-      else hi = mid;
+  for (uint32_t c = s_c0; c < nch; c++) {
+    const uint64_t c_beg = cs[c];
+    if (c_beg >= te) break;
+    const uint64_t i0 = uint64_t(c) * kRleChunk;
+    const uint32_t m = uint32_t(umin64(kRleChunk, r - i0));
+    for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) {
+      s_len[i] = lens[i0 + i];
+      s_val[i] = vals[i0 + i];
     }
-    dst[e] = values[lo];
+    if (threadIdx.x == 0) s_nlong = 0;
+    __syncthreads();
+    // run starts of the chunk: 8 consecutive runs per thread, block exclusive scan of the sums
+    constexpr uint32_t PER = kRleChunk / kThreads;
+    uint32_t l[PER];
+    uint64_t part = 0;
+#pragma unroll
+    for (int q = 0; q < int(PER); q++) {
+      const uint32_t i = threadIdx.x * PER + q;
+      l[q] = i < m ? s_len[i] : 0;
+      part += l[q];
+    }
+    uint64_t tot;
+    uint64_t st = c_beg + block_excl_sum_u64(part, s_tmp, &tot);
+#pragma unroll
+    for (int q = 0; q < int(PER); q++) {
+      const uint32_t i = threadIdx.x * PER + q;
+      const uint64_t a = st > tb ? st : tb, e = st + l[q];
+      const uint64_t b = e < te ? e : te;
+      if (i < m && a < b) {
+        const T v = s_val[i];
+        if (b - a <= 32) {
+          for (uint64_t x = a; x < b; x++) s_out[x - tb] = v;
+        } else {
+          const uint32_t slot = atomicAdd(&s_nlong, 1u);
+          s_long[slot][0] = uint32_t(a - tb);
+          s_long[slot][1] = uint32_t(b - tb);
+          s_long[slot][2] = uint32_t(v);
+        }
+      }
+      st = e;
+    }
+    __syncthreads();
+    for (uint32_t q = warp; q < s_nlong; q += kWarps) {  // long runs: a warp each
+      const uint32_t a = s_long[q][0], b = s_long[q][1];
+      const T v = T(s_long[q][2]);
+      for (uint32_t x = a + lane; x < b; x += 32) s_out[x] = v;
+    }
+    __syncthreads();
   }
+  T* dst = outp + uint64_t(p.k) * F + p.tin;
+  constexpr uint32_t EPV = 16 / sizeof(T);
+  const uint32_t nv = p.te / EPV;
+  for (uint32_t v = threadIdx.x; v < nv; v += blockDim.x)
+    stg_stream(reinterpret_cast<uint4*>(dst) + v, reinterpret_cast<const uint4*>(s_out)[v]);
+  for (uint32_t e = nv * EPV + threadIdx.x; e < p.te; e += blockDim.x) dst[e] = s_out[e];
 }
 
 cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
@@ -292,21 +384,23 @@ cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int 
   if (k1 <= k0) return cudaSuccess;
   const uint32_t TILE = kTileBytes / w;
   const uint32_t tpf = uint32_t(cdiv(F, TILE));
-  uint32_t* rs = nullptr;  // run starts, indexed k*F + i (i < r_k <= F_k): at most n entries
-  cudaError_t e = cudaMallocAsync(&rs, n * 4 + 64, st);
+  const uint32_t cpf = uint32_t(cdiv(F, kRleChunk));  // chunk slots per frame (r_k <= F_k <= F)
+  uint64_t* cs = nullptr;  // per chunk slot: sum of lengths, then the chunk's start position
+  cudaError_t e = cudaMallocAsync(&cs, uint64_t(k1 - k0) * cpf * 8 + 64, st);
   if (e != cudaSuccess) return e;
   const uint32_t tiles = (k1 - 1 - k0) * tpf + uint32_t(cdiv(frame_len(n, F, k1 - 1), TILE));
-  if (w == 4) {
-    timing_kernel_start(st);
-    rle_dscan_kernel<uint32_t><<<k1 - k0, 1024, 0, st>>>(in, n, F, k0, rs, sc, err);
-    rle_expand_kernel<uint32_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint32_t*>(out), n, F, tpf, k0, rs, sc, err);
-  } else {
-    timing_kernel_start(st);
-    rle_dscan_kernel<uint16_t><<<k1 - k0, 1024, 0, st>>>(in, n, F, k0, rs, sc, err);
-    rle_expand_kernel<uint16_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint16_t*>(out), n, F, tpf, k0, rs, sc, err);
-  }
+  timing_kernel_start(st);
+  const uint64_t dgrid = std::min<uint64_t>(cdiv(uint64_t(k1 - k0) * cpf, kWarps), 148 * 16);
+  rle_dsum_kernel<<<uint32_t(dgrid), kThreads, 0, st>>>(in, n, F, w, k0, k1, cpf, cs, sc, err);
+  rle_dscan2_kernel<<<k1 - k0, 1024, 0, st>>>(in, n, F, w, k0, cpf, cs, sc, err);
+  if (w == 4)
+    rle_paint_kernel<uint32_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint32_t*>(out), n, F, tpf, k0, cpf, cs,
+                                                           sc, err);
+  else
+    rle_paint_kernel<uint16_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint16_t*>(out), n, F, tpf, k0, cpf, cs,
+                                                           sc, err);
   e = cudaGetLastError();
-  cudaFreeAsync(rs, st);
+  cudaFreeAsync(cs, st);
   return e;
 }
 
