@@ -432,7 +432,7 @@ cswap_status decompress_range(Ctx* c, Lease& L, const uint8_t* in, void* out, ui
       c->launches += 3;  // count, scan, expand
       return cuda_status(launch_zvc_decompress(in, out, n, w, F, k0, k1, L.b->sc, L.epoch(), err, st), "zvc_decompress");
     case CSWAP_CODEC_RLE:
-      c->launches += 2;
+      c->launches += 4;  // chunk sums, chunk scan, runs, long-run fill
       return cuda_status(launch_rle_decompress(in, out, n, w, F, k0, k1, L.b->sc, L.epoch(), err, st), "rle_decompress");
     case CSWAP_CODEC_CSR:
       c->launches++;

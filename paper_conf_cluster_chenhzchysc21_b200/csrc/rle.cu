@@ -9,7 +9,7 @@
 // whole frame is counted; compress is therefore: count (run starts per tile + first start) ->
 // per-frame scan (run offsets, next run start after each tile, r_k) -> frame table -> emit.
 // Decompress: chunked scan of the lengths (chunk sums -> per-frame scan of the chunk sums), then
-// one CTA per output tile paints the runs overlapping it (see rle_paint_kernel).
+// run-parallel expansion (see rle_runs_kernel).
 #include "kernels.h"
 #include "tile_common.cuh"
 
@@ -201,14 +201,11 @@ cudaError_t launch_rle_compress(const void* in, uint64_t n, int w, uint64_t F, u
 // ------------------------------------------------------------------------------------------
 // one CTA per frame: validate, run start positions (frame-relative) into rs[k*F + i]
 // ---- decompress ------------------------------------------------------------------------------
-// The lengths of frame k are cut into chunks of kRleChunk runs.  (1) one CTA per chunk slot sums
+// The lengths of frame k are cut into chunks of kRleChunk runs.  (1) one warp per chunk slot sums
 // its chunk's lengths; (2) one CTA per frame validates the frame and scans the chunk sums into
-// chunk start positions; (3) one CTA per output tile finds the chunk holding its first element
-// (32-ary search over the frame's chunk starts), then for each chunk overlapping the tile scans
-// the chunk's lengths in shared memory into run starts and paints every run's clipped range
-// into a shared-memory copy of the tile (short runs by one thread, runs longer than 32 elements
-// by a whole warp), and stores the tile with 16-byte stores.  Traffic: lengths twice (the
-// second read mostly from L2), values once, output once.
+// chunk start positions; (3) rle_runs_kernel expands the runs of each chunk straight into the
+// output (run-parallel; long runs go to a piece list); (4) rle_fill_kernel fills the pieces.
+// Traffic: lengths twice, values once, output once.
 constexpr uint32_t kRleChunk = 1024;
 
 __device__ __forceinline__ bool rle_frame_header(const uint8_t* in, uint64_t fstart, uint64_t fb, uint64_t Fk, int w,
@@ -222,7 +219,9 @@ __device__ __forceinline__ bool rle_frame_header(const uint8_t* in, uint64_t fst
 // one warp per chunk slot, grid-stride (most slots of a frame are empty when runs are long)
 __global__ void __launch_bounds__(kThreads) rle_dsum_kernel(const uint8_t* __restrict__ in, uint64_t n, uint64_t F,
                                                             int w, uint32_t k0, uint32_t k1, uint32_t cpf,
-                                                            uint64_t* csum, Scratch sc, uint32_t* err) {
+                                                            uint64_t* csum, uint32_t* npieces, Scratch sc,
+                                                            uint32_t* err) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) *npieces = 0;  // rle_runs_kernel appends long-run pieces
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const int lane = threadIdx.x & 31;
   const uint64_t slots = uint64_t(k1 - k0) * cpf;
@@ -284,123 +283,139 @@ __global__ void __launch_bounds__(1024) rle_dscan2_kernel(const uint8_t* __restr
   if (threadIdx.x == 0 && carry != Fk) set_error(err, kErrCorrupt);
 }
 
+// Run-parallel expansion: one CTA per chunk slot (grid-stride), 8 warps x 128 consecutive runs.
+// Lane l of a warp holds runs l, 32+l, 64+l, 96+l, so one store instruction writes 32
+// consecutive runs' elements (coalesced for the short runs that dominate iid ReLU data).  Runs of
+// 33..kLongRun elements are filled by the whole warp; longer runs are cut into kPiece-element
+// pieces appended to a global list that rle_fill_kernel spreads over the grid (one run may
+// cover a whole frame).
+constexpr uint32_t kLongRun = 4096, kPiece = 8192;
+struct RlePiece {
+  uint64_t start;  // element index in the tensor
+  uint32_t len, value;
+};
+
 template <typename T>
-__global__ void __launch_bounds__(kThreads) rle_paint_kernel(const uint8_t* __restrict__ in, T* __restrict__ outp,
-                                                             uint64_t n, uint64_t F, uint32_t tpf, uint32_t k0,
-                                                             uint32_t cpf, const uint64_t* __restrict__ cstart,
-                                                             Scratch sc, uint32_t* err) {
-  using G = TileGeom<T>;
-  __shared__ __align__(16) T s_out[G::TILE];
-  __shared__ uint32_t s_len[kRleChunk];
-  __shared__ T s_val[kRleChunk];
-  __shared__ uint64_t s_tmp[33];
-  __shared__ uint32_t s_long[G::TILE / 33 + 2][3];  // runs longer than 32 elements inside the tile: (a, b, value)
-  __shared__ uint32_t s_nlong, s_c0;
+__global__ void __launch_bounds__(kThreads) rle_runs_kernel(const uint8_t* __restrict__ in, T* __restrict__ outp,
+                                                            uint64_t n, uint64_t F, uint32_t k0, uint32_t k1,
+                                                            uint32_t cpf, const uint64_t* __restrict__ cstart,
+                                                            RlePiece* pieces, uint32_t* npieces, uint64_t cap,
+                                                            Scratch sc, uint32_t* err) {
+  __shared__ uint64_t s_wtot[kWarps];
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
-  const uint32_t t = blockIdx.x + k0 * tpf;
-  const TilePos p = tile_pos<T>(t, n, F, tpf);
-  const uint64_t r = sc.aux3[p.k];
-  if (r == 0) return;
-  const uint32_t nch = uint32_t(cdiv(r, kRleChunk));
-  const uint64_t* cs = cstart + uint64_t(p.k - k0) * cpf;
-  const uint32_t* lens = reinterpret_cast<const uint32_t*>(in + sc.aux[p.k] + 16);
-  const T* vals = reinterpret_cast<const T*>(in + sc.aux[p.k] + 16 + a16(4 * r));
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint64_t tb = p.tin, te = p.tin + p.te;
-  if (warp == 0) {  // last chunk with start <= tb (chunk 0 starts at 0)
-    uint32_t lo = 0, hi = nch;
-    while (hi - lo > 1) {
-      const uint32_t span = hi - lo;
-      const uint32_t probe = lo + uint32_t((uint64_t(span) * lane) / 32);
-      const uint32_t m = __ballot_sync(0xffffffffu, cs[probe] <= tb);
-      const int last = 31 - __clz(m);
-      const uint32_t nlo = lo + uint32_t((uint64_t(span) * last) / 32);
-      const uint32_t nhi = last == 31 ? hi : lo + uint32_t((uint64_t(span) * (last + 1)) / 32);
-      lo = nlo;
-      hi = nhi > nlo ? nhi : nlo + 1;
-    }
-    if (lane == 0) s_c0 = lo;
-  }
-  __syncthreads();
-  for (uint32_t c = s_c0; c < nch; c++) {
-    const uint64_t c_beg = cs[c];
-    if (c_beg >= te) break;
+  const uint64_t slots = uint64_t(k1 - k0) * cpf;
+  for (uint64_t sl = blockIdx.x; sl < slots; sl += gridDim.x) {
+    const uint32_t k = k0 + uint32_t(sl / cpf), c = uint32_t(sl % cpf);
+    const uint64_t r = sc.aux3[k];  // validated by rle_dscan2 (0: corrupt frame)
     const uint64_t i0 = uint64_t(c) * kRleChunk;
+    if (i0 >= r) continue;  // uniform over the CTA
     const uint32_t m = uint32_t(umin64(kRleChunk, r - i0));
-    for (uint32_t i = threadIdx.x; i < m; i += blockDim.x) {
-      s_len[i] = lens[i0 + i];
-      s_val[i] = vals[i0 + i];
+    const uint32_t* lens = reinterpret_cast<const uint32_t*>(in + sc.aux[k] + 16) + i0;
+    const T* vals = reinterpret_cast<const T*>(in + sc.aux[k] + 16 + a16(4 * r)) + i0;
+    const uint32_t wb = warp * (kRleChunk / kWarps);
+    constexpr int Q = kRleChunk / kWarps / 32;
+    uint32_t L[Q];
+    T V[Q];
+    uint64_t S[Q], carry = 0;
+#pragma unroll
+    for (int q = 0; q < Q; q++) {
+      const uint32_t i = wb + q * 32 + lane;
+      L[q] = i < m ? lens[i] : 0u;
+      V[q] = i < m ? vals[i] : T(0);
     }
-    if (threadIdx.x == 0) s_nlong = 0;
+#pragma unroll
+    for (int q = 0; q < Q; q++) {  // exclusive prefix of the warp's runs, in run order
+      uint64_t inc = L[q];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += y;
+      }
+      S[q] = carry + inc - L[q];
+      carry += __shfl_sync(0xffffffffu, inc, 31);
+    }
+    if (lane == 0) s_wtot[warp] = carry;
     __syncthreads();
-    // run starts of the chunk: 8 consecutive runs per thread, block exclusive scan of the sums
-    constexpr uint32_t PER = kRleChunk / kThreads;
-    uint32_t l[PER];
-    uint64_t part = 0;
+    uint64_t wbase = cstart[sl];
+    for (int q = 0; q < warp; q++) wbase += s_wtot[q];
+    T* dst = outp + uint64_t(k) * F;
 #pragma unroll
-    for (int q = 0; q < int(PER); q++) {
-      const uint32_t i = threadIdx.x * PER + q;
-      l[q] = i < m ? s_len[i] : 0;
-      part += l[q];
-    }
-    uint64_t tot;
-    uint64_t st = c_beg + block_excl_sum_u64(part, s_tmp, &tot);
-#pragma unroll
-    for (int q = 0; q < int(PER); q++) {
-      const uint32_t i = threadIdx.x * PER + q;
-      const uint64_t a = st > tb ? st : tb, e = st + l[q];
-      const uint64_t b = e < te ? e : te;
-      if (i < m && a < b) {
-        const T v = s_val[i];
-        if (b - a <= 32) {
-          for (uint64_t x = a; x < b; x++) s_out[x - tb] = v;
+    for (int q = 0; q < Q; q++) {
+      const uint64_t st = wbase + S[q];
+      const uint32_t len = L[q];
+      const uint32_t sh = len <= 32 ? len : 0u;
+      const uint32_t mx = __reduce_max_sync(0xffffffffu, sh);
+      for (uint32_t e = 0; e < mx; e++)
+        if (e < sh) dst[st + e] = V[q];
+      uint32_t med = __ballot_sync(0xffffffffu, len > 32 && len <= kLongRun);
+      while (med) {
+        const int b = __ffs(med) - 1;
+        med &= med - 1;
+        const uint64_t s2 = __shfl_sync(0xffffffffu, st, b);
+        const uint32_t l2 = __shfl_sync(0xffffffffu, len, b);
+        const T v2 = T(__shfl_sync(0xffffffffu, uint32_t(V[q]), b));
+        for (uint32_t x = lane; x < l2; x += 32) dst[s2 + x] = v2;
+      }
+      if (len > kLongRun) {
+        const uint32_t np = (len + kPiece - 1) / kPiece;
+        const uint32_t idx = atomicAdd(npieces, np);
+        if (uint64_t(idx) + np > cap) {
+          set_error(err, kErrCorrupt);  // cannot happen for a valid container (cap >= n / kLongRun)
         } else {
-          const uint32_t slot = atomicAdd(&s_nlong, 1u);
-          s_long[slot][0] = uint32_t(a - tb);
-          s_long[slot][1] = uint32_t(b - tb);
-          s_long[slot][2] = uint32_t(v);
+          for (uint32_t p2 = 0; p2 < np; p2++)
+            pieces[idx + p2] = RlePiece{uint64_t(k) * F + st + uint64_t(p2) * kPiece,
+                                        (len - p2 * kPiece < kPiece ? len - p2 * kPiece : kPiece), uint32_t(V[q])};
         }
       }
-      st = e;
     }
-    __syncthreads();
-    for (uint32_t q = warp; q < s_nlong; q += kWarps) {  // long runs: a warp each
-      const uint32_t a = s_long[q][0], b = s_long[q][1];
-      const T v = T(s_long[q][2]);
-      for (uint32_t x = a + lane; x < b; x += 32) s_out[x] = v;
-    }
-    __syncthreads();
+    __syncthreads();  // s_wtot is rewritten by the next slot
   }
-  T* dst = outp + uint64_t(p.k) * F + p.tin;
-  constexpr uint32_t EPV = 16 / sizeof(T);
-  const uint32_t nv = p.te / EPV;
-  for (uint32_t v = threadIdx.x; v < nv; v += blockDim.x)
-    stg_stream(reinterpret_cast<uint4*>(dst) + v, reinterpret_cast<const uint4*>(s_out)[v]);
-  for (uint32_t e = nv * EPV + threadIdx.x; e < p.te; e += blockDim.x) dst[e] = s_out[e];
+}
+
+template <typename T>
+__global__ void __launch_bounds__(kThreads) rle_fill_kernel(T* __restrict__ outp, const RlePiece* pieces,
+                                                            const uint32_t* npieces) {
+  const uint32_t total = *npieces;
+  for (uint32_t p = blockIdx.x; p < total; p += gridDim.x) {
+    const RlePiece pc = pieces[p];
+    const T v = T(pc.value);
+    for (uint32_t x = threadIdx.x; x < pc.len; x += blockDim.x) outp[pc.start + x] = v;
+  }
 }
 
 cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
                                   uint32_t k1, const Scratch& sc, uint32_t /*epoch*/, uint32_t* err, cudaStream_t st) {
   if (k1 <= k0) return cudaSuccess;
-  const uint32_t TILE = kTileBytes / w;
-  const uint32_t tpf = uint32_t(cdiv(F, TILE));
   const uint32_t cpf = uint32_t(cdiv(F, kRleChunk));  // chunk slots per frame (r_k <= F_k <= F)
-  uint64_t* cs = nullptr;  // per chunk slot: sum of lengths, then the chunk's start position
-  cudaError_t e = cudaMallocAsync(&cs, uint64_t(k1 - k0) * cpf * 8 + 64, st);
+  const uint64_t slots = uint64_t(k1 - k0) * cpf;
+  const uint64_t elems = umin64(n, uint64_t(k1) * F) - uint64_t(k0) * F;
+  const uint64_t cap = elems / kLongRun + (elems / kPiece) + 2 * (k1 - k0) + 8;  // pieces
+  // one allocation: chunk sums / starts | piece counter | pieces
+  uint8_t* tmp = nullptr;
+  const uint64_t off_cnt = a16(slots * 8), off_pc = off_cnt + 16;
+  cudaError_t e = cudaMallocAsync(&tmp, off_pc + cap * sizeof(RlePiece), st);
   if (e != cudaSuccess) return e;
-  const uint32_t tiles = (k1 - 1 - k0) * tpf + uint32_t(cdiv(frame_len(n, F, k1 - 1), TILE));
+  uint64_t* cs = reinterpret_cast<uint64_t*>(tmp);
+  uint32_t* cnt = reinterpret_cast<uint32_t*>(tmp + off_cnt);
+  RlePiece* pcs = reinterpret_cast<RlePiece*>(tmp + off_pc);
   timing_kernel_start(st);
-  const uint64_t dgrid = std::min<uint64_t>(cdiv(uint64_t(k1 - k0) * cpf, kWarps), 148 * 16);
-  rle_dsum_kernel<<<uint32_t(dgrid), kThreads, 0, st>>>(in, n, F, w, k0, k1, cpf, cs, sc, err);
+  const uint64_t dgrid = std::min<uint64_t>(cdiv(slots, kWarps), 148 * 16);
+  rle_dsum_kernel<<<uint32_t(dgrid), kThreads, 0, st>>>(in, n, F, w, k0, k1, cpf, cs, cnt, sc, err);
   rle_dscan2_kernel<<<k1 - k0, 1024, 0, st>>>(in, n, F, w, k0, cpf, cs, sc, err);
-  if (w == 4)
-    rle_paint_kernel<uint32_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint32_t*>(out), n, F, tpf, k0, cpf, cs,
-                                                           sc, err);
-  else
-    rle_paint_kernel<uint16_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint16_t*>(out), n, F, tpf, k0, cpf, cs,
-                                                           sc, err);
+  const uint32_t rgrid = uint32_t(std::min<uint64_t>(slots, 148 * 8));
+  const uint32_t fgrid = 148 * 4;
+  if (w == 4) {
+    rle_runs_kernel<uint32_t><<<rgrid, kThreads, 0, st>>>(in, static_cast<uint32_t*>(out), n, F, k0, k1, cpf, cs,
+                                                          pcs, cnt, cap, sc, err);
+    rle_fill_kernel<uint32_t><<<fgrid, kThreads, 0, st>>>(static_cast<uint32_t*>(out), pcs, cnt);
+  } else {
+    rle_runs_kernel<uint16_t><<<rgrid, kThreads, 0, st>>>(in, static_cast<uint16_t*>(out), n, F, k0, k1, cpf, cs,
+                                                          pcs, cnt, cap, sc, err);
+    rle_fill_kernel<uint16_t><<<fgrid, kThreads, 0, st>>>(static_cast<uint16_t*>(out), pcs, cnt);
+  }
   e = cudaGetLastError();
-  cudaFreeAsync(cs, st);
+  cudaFreeAsync(tmp, st);
   return e;
 }
 
