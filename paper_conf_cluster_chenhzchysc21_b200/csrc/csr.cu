@@ -23,7 +23,25 @@ __global__ void __launch_bounds__(kThreads) csr_count_kernel(const T* __restrict
   const TilePos p = tile_pos<T>(t, n, F, tpf);
   const T* src = in + uint64_t(p.k) * F + p.tin;
   uint32_t c = 0;
-  for (uint32_t e = threadIdx.x; e < p.te; e += blockDim.x) c += src[e] != 0;
+  if (p.te == G::TILE) {  // full tile: 16-byte loads, all in flight
+    constexpr int V = G::TILE * int(sizeof(T)) / 16 / kThreads;
+    const uint4* s4 = reinterpret_cast<const uint4*>(src);
+    uint4 q[V];
+#pragma unroll
+    for (int i = 0; i < V; i++) q[i] = __ldg(s4 + threadIdx.x + i * kThreads);
+#pragma unroll
+    for (int i = 0; i < V; i++) {
+      if constexpr (sizeof(T) == 4) {
+        c += (q[i].x != 0) + (q[i].y != 0) + (q[i].z != 0) + (q[i].w != 0);
+      } else {
+        const uint32_t w4[4] = {q[i].x, q[i].y, q[i].z, q[i].w};
+#pragma unroll
+        for (int h = 0; h < 4; h++) c += ((w4[h] & 0xFFFFu) != 0) + ((w4[h] >> 16) != 0);
+      }
+    }
+  } else {
+    for (uint32_t e = threadIdx.x; e < p.te; e += blockDim.x) c += src[e] != 0;
+  }
   c = block_sum_u32(c, s_tmp);
   if (threadIdx.x == 0) sc.tbuf[t] = c;
 }
@@ -66,10 +84,20 @@ __global__ void __launch_bounds__(kThreads) csr_emit_kernel(const T* __restrict_
   const T* src = in + uint64_t(p.k) * F + p.tin;
   const uint32_t lt = (1u << lane) - 1u;
   // pass 1: per-warp counts (warp w owns elements [w*PER_WARP, (w+1)*PER_WARP) as rows of 32)
+  // rows are loaded 8 at a time before their ballots (independent loads in flight)
+  constexpr int B = 8;
+  const bool full = p.te == G::TILE;
   uint32_t cnt = 0;
-  for (int m = 0; m < G::ROWS; m++) {
-    const uint32_t e = warp * G::PER_WARP + 32 * m + lane;
-    cnt += __popc(__ballot_sync(0xffffffffu, e < p.te && src[e] != 0));
+#pragma unroll 1
+  for (int m0 = 0; m0 < G::ROWS; m0 += B) {
+    T v[B];
+#pragma unroll
+    for (int u = 0; u < B; u++) {
+      const uint32_t e = warp * G::PER_WARP + 32 * (m0 + u) + lane;
+      v[u] = (full || e < p.te) ? src[e] : T(0);
+    }
+#pragma unroll
+    for (int u = 0; u < B; u++) cnt += __popc(__ballot_sync(0xffffffffu, v[u] != 0));
   }
   if (lane == 0) s_wcnt[warp] = cnt;
   __syncthreads();
@@ -91,19 +119,36 @@ __global__ void __launch_bounds__(kThreads) csr_emit_kernel(const T* __restrict_
   const uint64_t tile_off = sc.tbuf[t];
   // pass 2: emit (col, value) at rank; row_ptr[r+1] at every row's last element
   uint64_t pre = tile_off + s_wcnt[warp];
-  for (int m = 0; m < G::ROWS; m++) {
-    const uint32_t e = warp * G::PER_WARP + 32 * m + lane;
-    const bool in_tile = e < p.te;
-    const T v = in_tile ? src[e] : T(0);
-    const uint32_t b = __ballot_sync(0xffffffffu, v != 0);
-    const uint64_t rank = pre + __popc(b & lt);
-    const uint64_t pos = p.tin + e;  // frame position
-    if (v != 0) {
-      col_idx[rank] = uint32_t(pos % C);
-      values[rank] = v;
+  // column / row of tile element e: x = (tin mod C) + e; power-of-two C by mask and shift
+  const uint32_t cbase = uint32_t(p.tin % C);
+  const uint64_t row0 = p.tin / C;
+  const bool pow2 = (C & (C - 1)) == 0;
+  const int csh = __ffs(int(C)) - 1;
+#pragma unroll 1
+  for (int m0 = 0; m0 < G::ROWS; m0 += B) {
+    T vb[B];
+#pragma unroll
+    for (int u = 0; u < B; u++) {
+      const uint32_t e = warp * G::PER_WARP + 32 * (m0 + u) + lane;
+      vb[u] = (full || e < p.te) ? src[e] : T(0);
     }
-    if (in_tile && ((pos + 1) % C == 0 || pos + 1 == Fk)) row_ptr[pos / C + 1] = uint32_t(rank + (v != 0));
-    pre += __popc(b);
+#pragma unroll
+    for (int u = 0; u < B; u++) {
+      const uint32_t e = warp * G::PER_WARP + 32 * (m0 + u) + lane;
+      const T v = vb[u];
+      const uint32_t b = __ballot_sync(0xffffffffu, v != 0);
+      const uint64_t rank = pre + __popc(b & lt);
+      const uint32_t x = cbase + e;
+      const uint32_t ro = pow2 ? x >> csh : x / C;
+      const uint32_t col = x - ro * C;
+      if (v != 0) {
+        col_idx[rank] = col;
+        values[rank] = v;
+      }
+      if ((full || e < p.te) && (col == C - 1 || p.tin + e + 1 == Fk))
+        row_ptr[row0 + ro + 1] = uint32_t(rank + (v != 0));
+      pre += __popc(b);
+    }
   }
   if (tid == 0 && p.j == 0) row_ptr[0] = 0;
   if (tid == kThreads - 1 && p.tin + p.te == Fk) {  // last tile of the frame: section pads

@@ -111,10 +111,19 @@ __global__ void __launch_bounds__(kThreads) rle_emit_kernel(const T* __restrict_
     if (f) wpos[cnt + __popc(b & lt)] = uint16_t(e);
     cnt += __popc(b);
   }
-  if (lane == 0) s_wcnt[warp] = cnt;
+  __shared__ uint32_t s_wfirst[kWarps], s_wnext[kWarps];
+  __syncwarp();
+  if (lane == 0) {
+    s_wcnt[warp] = cnt;
+    s_wfirst[warp] = cnt ? uint32_t(wpos[0]) : 0xFFFFFFFFu;
+  }
   __syncthreads();
-  if (tid == 0) {
-    uint32_t a = 0;
+  if (tid == 0) {  // run offset of each warp's list, and the first run start after each warp
+    uint32_t a = 0, nx = 0xFFFFFFFFu;
+    for (int w = kWarps - 1; w >= 0; w--) {
+      s_wnext[w] = nx;
+      if (s_wfirst[w] != 0xFFFFFFFFu) nx = s_wfirst[w];
+    }
     for (int w = 0; w < kWarps; w++) {
       const uint32_t x = s_wcnt[w];
       s_wcnt[w] = a;
@@ -123,29 +132,19 @@ __global__ void __launch_bounds__(kThreads) rle_emit_kernel(const T* __restrict_
     s_wcnt[kWarps] = a;
   }
   __syncthreads();
-  const uint32_t total = s_wcnt[kWarps];
   const uint64_t run_off = sc.tbuf[t];
   const uint64_t next_start = sc.tbuf2[t];
   const uint64_t r_k = sc.aux3[p.k];
   const uint64_t fstart = sc.aux[p.k];
-  uint32_t* lengths = reinterpret_cast<uint32_t*>(out + fstart + 16);
-  uint8_t* values = out + fstart + 16 + a16(4 * r_k);
-  // gather the warp lists into one ordered sequence: run q of the tile is in warp w's list at
-  // q - s_wcnt[w]; write length and value of every run starting in this tile
-  for (uint32_t q = tid; q < total; q += kThreads) {
-    int w = 0;
-    while (w + 1 < kWarps && s_wcnt[w + 1] <= q) w++;
-    const uint32_t pos = s_bpos[w * G::PER_WARP + (q - s_wcnt[w])];
-    uint64_t end;
-    if (q + 1 < total) {
-      int w2 = w;
-      while (w2 + 1 < kWarps && s_wcnt[w2 + 1] <= q + 1) w2++;
-      end = p.tin + s_bpos[w2 * G::PER_WARP + (q + 1 - s_wcnt[w2])];
-    } else {
-      end = next_start;
-    }
-    lengths[run_off + q] = uint32_t(end - (p.tin + pos));
-    reinterpret_cast<T*>(values)[run_off + q] = s_x[pos];
+  uint32_t* lengths = reinterpret_cast<uint32_t*>(out + fstart + 16) + run_off + s_wcnt[warp];
+  T* values = reinterpret_cast<T*>(out + fstart + 16 + a16(4 * r_k)) + run_off + s_wcnt[warp];
+  // each warp writes the runs starting in its slab: consecutive lanes, consecutive runs
+  const uint64_t after = s_wnext[warp] != 0xFFFFFFFFu ? p.tin + s_wnext[warp] : next_start;
+  for (uint32_t q = lane; q < cnt; q += 32) {
+    const uint32_t pos = wpos[q];
+    const uint64_t end = q + 1 < cnt ? p.tin + wpos[q + 1] : after;
+    lengths[q] = uint32_t(end - (p.tin + pos));
+    values[q] = s_x[pos];
   }
   if (tid == 0 && p.j == 0) {  // sub-header {u32 r, 12 zero bytes}
     uint32_t* h = reinterpret_cast<uint32_t*>(out + fstart);
