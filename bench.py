@@ -460,16 +460,26 @@ def _decision_accuracy(C, torch, items, dtype, chosen) -> dict:
 
 def _e2e(args, C, torch, tensors, outs, sizes, dtype, w, dist, world, stream) -> dict:
     """Same metric through the public API with HOST inputs: per step the 12 inputs are copied
-    H2D from pinned host memory, swapped out and back in, and 16 bytes of every restored
-    tensor are read back D2H."""
+    H2D from pinned host memory (input i+1's copy overlapping tensor i's swap-out), swapped out
+    and back in, and 16 bytes of every restored tensor are read back D2H."""
     hosts = [t.cpu().pin_memory() for t in tensors]
     probe_back = torch.empty(len(tensors), 4, dtype=torch.int32).pin_memory()
     steps = max(2, min(args.steps, 5))
+    # the input copies run on their own stream, one event per tensor, so the H2D of input i+1
+    # overlaps the swap-out (compress + D2H) of tensor i: PCIe is full duplex
+    cs = torch.cuda.Stream()
+    landed = [torch.cuda.Event() for _ in tensors]
 
     def one():
-        for hst, t in zip(hosts, tensors):
-            t.copy_(hst, non_blocking=True)
-        hs = [C.swap_out(t, n, dtype, C.AUTO) for t, n in zip(tensors, sizes)]
+        cs.wait_stream(stream)
+        with torch.cuda.stream(cs):
+            for hst, t, e in zip(hosts, tensors, landed):
+                t.copy_(hst, non_blocking=True)
+                e.record(cs)
+        hs = []
+        for t, n, e in zip(tensors, sizes, landed):
+            stream.wait_event(e)
+            hs.append(C.swap_out(t, n, dtype, C.AUTO))
         for o, h in zip(reversed(outs), reversed(hs)):
             h.swap_in(o)
         for i, o in enumerate(outs):

@@ -194,6 +194,14 @@ const char* cswap_status_string(cswap_status s);
 const char* cswap_last_error(void);
 /* Number of kernels this library launched since init (for bench accounting). */
 uint64_t cswap_kernel_launches(void);
+/* Launch groups (the kernels of one compress, one decompress, one swap-in frame group) run as
+ * CUDA graphs: captured on a per-thread stream and replayed on the caller's stream, the
+ * executable graph cached per (thread, stream, group kind) and updated in place.  Reason: while a
+ * copy engine streams over PCIe, a plainly launched kernel boundary costs 5-10 us on B200, a
+ * boundary inside a graph 0.5 us.  Environment CSWAP_GRAPHS=0 launches plainly.
+ * Writes the number of graph launches and of instantiations since init (either pointer may be
+ * NULL). */
+void cswap_graph_stats(uint64_t* launches, uint64_t* instantiations);
 
 #ifdef __cplusplus
 }

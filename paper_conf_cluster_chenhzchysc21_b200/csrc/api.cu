@@ -15,6 +15,7 @@
 #include <map>
 #include <mutex>
 #include <string>
+#include <tuple>
 #include <unordered_map>
 #include <vector>
 
@@ -167,6 +168,8 @@ struct Ctx {
   PinnedPool pinned;
   uint32_t* dev_err = nullptr;  // err word for cswap_decompress(err = NULL)
   std::atomic<uint64_t> launches{0};
+  std::atomic<uint64_t> graph_launches{0}, graph_instantiations{0};
+  uint64_t gen = 0;  // distinguishes this context from earlier init/shutdown cycles (graph caches)
   // kernel timing (cswap_set_kernel_timing)
   std::atomic<bool> timing{false};
   std::mutex tm_m;
@@ -219,6 +222,116 @@ struct Timer {
 void cswap::timing_kernel_start(cudaStream_t) {
   if (t_pending) t_pending->start_now();
 }
+
+namespace {
+
+// ---------------------------------------------------------------------------------------------
+// launch groups as CUDA graphs
+// ---------------------------------------------------------------------------------------------
+// While a copy engine streams over PCIe (the swap pipeline always has one running), every
+// kernel boundary of plainly launched kernels costs 5-10 us (tools/launch_probe.py on B200:
+// 2.1 us per boundary alone, 9.6 us during a D2H, 5.5 us during an H2D), while the boundaries
+// inside an uploaded graph cost 0.5 us in all three cases.  So the kernels of one launch group
+// (one compress; one swap-in frame group; one decompress) are captured on a per-thread capture
+// stream and replayed on the caller's stream as one graph.  The executable graph is cached per
+// (thread, stream, group key) and updated in place (cudaGraphExecUpdate) with the new pointers /
+// sizes; it is re-instantiated only when the topology changes.  CSWAP_GRAPHS=0 launches plainly.
+std::atomic<uint64_t> g_gen{0};
+
+bool graphs_enabled() {
+  static int on = -1;
+  if (on < 0) {
+    const char* e = getenv("CSWAP_GRAPHS");
+    on = (e && e[0] == '0') ? 0 : 1;
+  }
+  return on == 1;
+}
+
+struct GraphCache {
+  struct Ent {
+    cudaGraphExec_t exec = nullptr;
+    uint64_t last = 0;
+  };
+  std::map<std::tuple<cudaStream_t, uint64_t>, Ent> m;
+  cudaStream_t cap = nullptr;
+  uint64_t gen = 0, tick = 0;
+  void reset(uint64_t g) {
+    if (gen == g_gen.load()) {  // the context these belong to is still alive
+      for (auto& kv : m)
+        if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
+      if (cap) cudaStreamDestroy(cap);
+    }
+    m.clear();
+    cap = nullptr;
+    gen = g;
+  }
+};
+thread_local GraphCache t_gc;
+constexpr size_t kGraphCacheMax = 64;
+
+// Run fn(stream) — a function that only enqueues kernels — as one graph on st (or directly on st
+// when graphs are disabled).  A pending kernel timer gets its start event on st right before the
+// graph launch (timing events cannot be recorded inside a capture).
+template <class Fn>
+cswap_status run_group(Ctx* c, cudaStream_t st, uint64_t key, Fn&& fn) {
+  if (!graphs_enabled()) return fn(st);
+  GraphCache& g = t_gc;
+  if (g.gen != c->gen) g.reset(c->gen);
+  if (!g.cap && cudaStreamCreateWithFlags(&g.cap, cudaStreamNonBlocking) != cudaSuccess)
+    return fail(CSWAP_ERR_CUDA, "capture stream create failed");
+  if (cudaStreamBeginCapture(g.cap, cudaStreamCaptureModeRelaxed) != cudaSuccess)
+    return fail(CSWAP_ERR_CUDA, "begin capture failed: %s", cudaGetErrorString(cudaGetLastError()));
+  Timer* pending = t_pending;
+  t_pending = nullptr;
+  cswap_status s = fn(g.cap);
+  t_pending = pending;
+  cudaGraph_t graph = nullptr;
+  const cudaError_t e = cudaStreamEndCapture(g.cap, &graph);
+  if (s != CSWAP_OK || e != cudaSuccess) {
+    if (graph) cudaGraphDestroy(graph);
+    cudaGetLastError();
+    return s != CSWAP_OK ? s : fail(CSWAP_ERR_CUDA, "capture failed: %s", cudaGetErrorString(e));
+  }
+  auto& ent = g.m[std::make_tuple(st, key)];
+  ent.last = ++g.tick;
+  if (ent.exec) {
+    cudaGraphExecUpdateResultInfo info;
+    if (cudaGraphExecUpdate(ent.exec, graph, &info) != cudaSuccess) {
+      cudaGetLastError();
+      cudaGraphExecDestroy(ent.exec);
+      ent.exec = nullptr;
+    }
+  }
+  if (!ent.exec) {
+    if (cudaGraphInstantiate(&ent.exec, graph, 0) != cudaSuccess) {
+      ent.exec = nullptr;
+      cudaGraphDestroy(graph);
+      return fail(CSWAP_ERR_CUDA, "graph instantiate failed: %s", cudaGetErrorString(cudaGetLastError()));
+    }
+    c->graph_instantiations++;
+  }
+  cudaGraphDestroy(graph);
+  if (pending) pending->start_now();
+  if (cudaGraphLaunch(ent.exec, st) != cudaSuccess)
+    return fail(CSWAP_ERR_CUDA, "graph launch failed: %s", cudaGetErrorString(cudaGetLastError()));
+  c->graph_launches++;
+  if (g.m.size() > kGraphCacheMax) {  // evict the least recently used (freed once it has run)
+    auto lru = g.m.begin();
+    for (auto it = g.m.begin(); it != g.m.end(); ++it)
+      if (it->second.last < lru->second.last) lru = it;
+    if (lru->second.exec) cudaGraphExecDestroy(lru->second.exec);
+    g.m.erase(lru);
+  }
+  return CSWAP_OK;
+}
+
+// group keys: kind << 16 | codec << 8 | dtype
+constexpr uint64_t kGrpCompress = 1, kGrpSwapIn = 2, kGrpSwapInFirst = 3, kGrpDecompress = 4;
+inline uint64_t group_key(uint64_t kind, int codec, int dtype) {
+  return kind << 16 | uint64_t(codec) << 8 | uint64_t(dtype);
+}
+
+}  // namespace
 
 namespace {
 
@@ -386,20 +499,29 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       Lease L(*c, st, tiles, aux);
       TRY(L.status);
       c->launches += 2;  // accumulator zero fill + persistent compress
-      return cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, L.b->sc, L.epoch(), dtype, st), "zvc_compress");
+      const uint32_t ep = L.epoch();
+      return run_group(c, st, group_key(kGrpCompress, codec, dtype), [&](cudaStream_t gs) {
+        return cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, L.b->sc, ep, dtype, gs), "zvc_compress");
+      });
     }
     case CSWAP_CODEC_RLE: {
       Lease L(*c, st, rle_tiles(n, w, F) + 2, uint64_t(K) + 2);
       TRY(L.status);
       c->launches += 4;
-      return cuda_status(launch_rle_compress(in, n, w, F, out, out_size, L.b->sc, L.epoch(), dtype, st), "rle_compress");
+      const uint32_t ep = L.epoch();
+      return run_group(c, st, group_key(kGrpCompress, codec, dtype), [&](cudaStream_t gs) {
+        return cuda_status(launch_rle_compress(in, n, w, F, out, out_size, L.b->sc, ep, dtype, gs), "rle_compress");
+      });
     }
     case CSWAP_CODEC_CSR: {
       Lease L(*c, st, rle_tiles(n, w, F) + 2, uint64_t(K) + 2);
       TRY(L.status);
       c->launches += 4;
-      return cuda_status(launch_csr_compress(in, n, w, F, f.csr_row, out, out_size, L.b->sc, L.epoch(), dtype, st),
-                         "csr_compress");
+      const uint32_t ep = L.epoch();
+      return run_group(c, st, group_key(kGrpCompress, codec, dtype), [&](cudaStream_t gs) {
+        return cuda_status(launch_csr_compress(in, n, w, F, f.csr_row, out, out_size, L.b->sc, ep, dtype, gs),
+                           "csr_compress");
+      });
     }
     case CSWAP_CODEC_LZ4: {
       const uint64_t blocks = lz4_scratch_bytes(n, w, F, f.lz4_block);
@@ -411,8 +533,10 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
         Lease L(*c, st, bidx + 2, uint64_t(K) + 2);
         TRY(L.status);
         c->launches += 3;
-        s = cuda_status(launch_lz4_compress(in, n, w, F, f.lz4_block, out, out_size, slots, L.b->sc, dtype, st),
-                        "lz4_compress");
+        s = run_group(c, st, group_key(kGrpCompress, codec, dtype), [&](cudaStream_t gs) {
+          return cuda_status(launch_lz4_compress(in, n, w, F, f.lz4_block, out, out_size, slots, L.b->sc, dtype, gs),
+                             "lz4_compress");
+        });
       }
       CU(cudaFreeAsync(slots, st));
       return s;
@@ -422,18 +546,21 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
 }
 
 // ---- decompress frames [k0, k1) (prep must have run in the same lease) -----------------------
+// `tmp`: caller-owned decode scratch (decompress_tmp_bytes), so the group allocates nothing and
+// can be captured as a graph
 cswap_status decompress_range(Ctx* c, Lease& L, const uint8_t* in, void* out, uint64_t n, int dtype, int codec,
-                              const cswap_format& f, uint32_t k0, uint32_t k1, uint32_t* err, cudaStream_t st) {
+                              const cswap_format& f, uint32_t k0, uint32_t k1, uint32_t* err, uint8_t* tmp,
+                              cudaStream_t st) {
   const int w = width(dtype);
   const uint64_t F = f.frame_elems;
   switch (codec) {
     case CSWAP_CODEC_NONE: return CSWAP_OK;  // handled by the caller (raw copy)
     case CSWAP_CODEC_ZVC:
       c->launches += 3;  // count, scan, expand
-      return cuda_status(launch_zvc_decompress(in, out, n, w, F, k0, k1, L.b->sc, L.epoch(), err, st), "zvc_decompress");
+      return cuda_status(launch_zvc_decompress(in, out, n, w, F, k0, k1, L.b->sc, 0, err, st), "zvc_decompress");
     case CSWAP_CODEC_RLE:
       c->launches += 4;  // chunk sums, chunk scan, runs, long-run fill
-      return cuda_status(launch_rle_decompress(in, out, n, w, F, k0, k1, L.b->sc, L.epoch(), err, st), "rle_decompress");
+      return cuda_status(launch_rle_decompress(in, out, n, w, F, k0, k1, L.b->sc, 0, err, tmp, st), "rle_decompress");
     case CSWAP_CODEC_CSR:
       c->launches++;
       return cuda_status(launch_csr_decompress(in, out, n, w, F, f.csr_row, k0, k1, L.b->sc, err, st), "csr_decompress");
@@ -443,6 +570,10 @@ cswap_status decompress_range(Ctx* c, Lease& L, const uint8_t* in, void* out, ui
                          "lz4_decompress");
     default: return fail(CSWAP_ERR_INVALID, "unknown codec %d", codec);
   }
+}
+
+uint64_t decompress_tmp_bytes(int codec, uint64_t n, const cswap_format& f, uint32_t k0, uint32_t k1) {
+  return codec == CSWAP_CODEC_RLE ? rle_decompress_tmp_bytes(n, f.frame_elems, k0, k1) : 0;
 }
 
 uint64_t decompress_tiles(uint64_t n, int w, const cswap_format& f) {
@@ -508,6 +639,11 @@ const char* cswap_last_error(void) { return g_err.c_str(); }
 
 uint64_t cswap_kernel_launches(void) { return g_ctx ? g_ctx->launches.load() : 0; }
 
+void cswap_graph_stats(uint64_t* launches, uint64_t* instantiations) {
+  if (launches) *launches = g_ctx ? g_ctx->graph_launches.load() : 0;
+  if (instantiations) *instantiations = g_ctx ? g_ctx->graph_instantiations.load() : 0;
+}
+
 cswap_status cswap_init(int device) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (g_ctx) {
@@ -517,6 +653,7 @@ cswap_status cswap_init(int device) {
   CU(cudaSetDevice(device));
   Ctx* c = new Ctx();
   c->device = device;
+  c->gen = ++g_gen;
   CU(cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device));
   CU(cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking));
   CU(cudaStreamCreateWithFlags(&c->s_h2d, cudaStreamNonBlocking));
@@ -650,18 +787,23 @@ cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uin
   // reads it); the word is merged into the caller's at the end
   uint32_t* e = L.b->sc.err;
   const uint8_t* inb = static_cast<const uint8_t*>(in);
-  c->launches += 2;
-  TRY(cuda_status(launch_prep(inb, in_size, codec, dtype, n, F, param_of(codec, f), L.b->sc, e, true, st), "prep"));
-  cswap_status s = CSWAP_OK;
-  if (n != 0) {
-    if (codec == CSWAP_CODEC_NONE) {
-      c->launches++;
-      s = cuda_status(launch_none_decompress(inb, d_out, n, w, F, L.b->sc, e, st), "none_decompress");
-    } else {
-      s = decompress_range(c, L, inb, d_out, n, dtype, codec, f, 0, K, e, st);
+  uint8_t* tmp = nullptr;
+  const uint64_t tmp_bytes = n ? decompress_tmp_bytes(codec, n, f, 0, K) : 0;
+  if (tmp_bytes) CU(cudaMallocAsync(&tmp, tmp_bytes, st));
+  c->launches += 2;  // prep, err merge (+ the codec's kernels)
+  cswap_status s = run_group(c, st, group_key(kGrpDecompress, codec, dtype), [&](cudaStream_t gs) {
+    TRY(cuda_status(launch_prep(inb, in_size, codec, dtype, n, F, param_of(codec, f), L.b->sc, e, true, gs), "prep"));
+    if (n != 0) {
+      if (codec == CSWAP_CODEC_NONE) {
+        c->launches++;
+        TRY(cuda_status(launch_none_decompress(inb, d_out, n, w, F, L.b->sc, e, gs), "none_decompress"));
+      } else {
+        TRY(decompress_range(c, L, inb, d_out, n, dtype, codec, f, 0, K, e, tmp, gs));
+      }
     }
-  }
-  TRY(cuda_status(launch_err_merge(e, user_err, st), "err_merge"));
+    return cuda_status(launch_err_merge(e, user_err, gs), "err_merge");
+  });
+  if (tmp) cudaFreeAsync(tmp, st);
   return s;
 }
 
@@ -914,19 +1056,31 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
         s = fail(CSWAP_ERR_CUDA, "prefetch copy failed");
         break;
       }
-      Timer tm(c, st);
-      if (k0 == 0) {
-        c->launches++;
-        s = cuda_status(launch_prep(staging, h->bytes, h->codec, h->dtype, n, F, param_of(h->codec, f), L.b->sc,
-                                    e_dev, true, st),
-                        "prep");
+      uint8_t* tmp = nullptr;
+      const uint64_t tmp_bytes = decompress_tmp_bytes(h->codec, n, f, k0, k1);
+      if (tmp_bytes && cudaMallocAsync(&tmp, tmp_bytes, st) != cudaSuccess) {
+        s = fail(CSWAP_ERR_NOMEM, "decode scratch");
+        break;
       }
-      if (s == CSWAP_OK) s = decompress_range(c, L, staging, d_out, n, h->dtype, h->codec, f, k0, k1, e_dev, st);
+      Timer tm(c, st);
+      const bool first = k0 == 0, last = k1 == K;
+      c->launches += (first ? 1 : 0) + (last ? 1 : 0);
+      s = run_group(c, st, group_key(first ? kGrpSwapInFirst : kGrpSwapIn, h->codec, h->dtype) | (last ? 1u << 20 : 0),
+                    [&](cudaStream_t gs) {
+                      if (first)
+                        TRY(cuda_status(launch_prep(staging, h->bytes, h->codec, h->dtype, n, F,
+                                                    param_of(h->codec, f), L.b->sc, e_dev, true, gs),
+                                        "prep"));
+                      TRY(decompress_range(c, L, staging, d_out, n, h->dtype, h->codec, f, k0, k1, e_dev, tmp, gs));
+                      // the last group folds the device error word into the handle's pinned slot
+                      if (last) TRY(cuda_status(launch_err_merge(e_dev, h->err_slot(), gs), "err_merge"));
+                      return CSWAP_OK;
+                    });
+      if (tmp) cudaFreeAsync(tmp, st);
       const uint64_t raw = (std::min<uint64_t>(n, uint64_t(k1) * F) - uint64_t(k0) * F) * w;
       tm.commit(h->codec, 1, raw, end - off);
       off = end;
     }
-    if (s == CSWAP_OK) s = cuda_status(launch_err_merge(e_dev, h->err_slot(), st), "err_merge");
   }
   cudaFreeAsync(staging, st);
   cudaEventRecord(h->ev_in, st);

@@ -41,8 +41,10 @@ cudaError_t launch_zvc_decompress(const uint8_t* in, void* out, uint64_t n, int 
 uint32_t rle_tiles(uint64_t n, int w, uint64_t F);
 cudaError_t launch_rle_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
                                 const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st);
+uint64_t rle_decompress_tmp_bytes(uint64_t n, uint64_t F, uint32_t k0, uint32_t k1);
 cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
-                                  uint32_t k1, const Scratch& sc, uint32_t epoch, uint32_t* err, cudaStream_t st);
+                                  uint32_t k1, const Scratch& sc, uint32_t epoch, uint32_t* err, uint8_t* tmp,
+                                  cudaStream_t st);
 
 // csr.cu
 cudaError_t launch_csr_compress(const void* in, uint64_t n, int w, uint64_t F, uint32_t C, uint8_t* out,

@@ -383,18 +383,34 @@ __global__ void __launch_bounds__(kThreads) rle_fill_kernel(T* __restrict__ outp
   }
 }
 
-cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
-                                  uint32_t k1, const Scratch& sc, uint32_t /*epoch*/, uint32_t* err, cudaStream_t st) {
-  if (k1 <= k0) return cudaSuccess;
+// scratch of one decode of frames [k0, k1): chunk sums / starts | piece counter | pieces
+static void rle_dtmp_layout(uint64_t n, uint64_t F, uint32_t k0, uint32_t k1, uint64_t* slots, uint64_t* cap,
+                            uint64_t* off_cnt, uint64_t* off_pc, uint64_t* bytes) {
   const uint32_t cpf = uint32_t(cdiv(F, kRleChunk));  // chunk slots per frame (r_k <= F_k <= F)
-  const uint64_t slots = uint64_t(k1 - k0) * cpf;
+  *slots = uint64_t(k1 - k0) * cpf;
   const uint64_t elems = umin64(n, uint64_t(k1) * F) - uint64_t(k0) * F;
-  const uint64_t cap = elems / kLongRun + (elems / kPiece) + 2 * (k1 - k0) + 8;  // pieces
-  // one allocation: chunk sums / starts | piece counter | pieces
-  uint8_t* tmp = nullptr;
-  const uint64_t off_cnt = a16(slots * 8), off_pc = off_cnt + 16;
-  cudaError_t e = cudaMallocAsync(&tmp, off_pc + cap * sizeof(RlePiece), st);
-  if (e != cudaSuccess) return e;
+  *cap = elems / kLongRun + (elems / kPiece) + 2 * (k1 - k0) + 8;  // pieces
+  *off_cnt = a16(*slots * 8);
+  *off_pc = *off_cnt + 16;
+  *bytes = *off_pc + *cap * sizeof(RlePiece);
+}
+
+uint64_t rle_decompress_tmp_bytes(uint64_t n, uint64_t F, uint32_t k0, uint32_t k1) {
+  if (k1 <= k0) return 0;
+  uint64_t slots, cap, off_cnt, off_pc, bytes;
+  rle_dtmp_layout(n, F, k0, k1, &slots, &cap, &off_cnt, &off_pc, &bytes);
+  return bytes;
+}
+
+// `tmp` (rle_decompress_tmp_bytes) is owned by the caller, so the launch group allocates nothing
+// and can be captured into a graph
+cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,
+                                  uint32_t k1, const Scratch& sc, uint32_t /*epoch*/, uint32_t* err, uint8_t* tmp,
+                                  cudaStream_t st) {
+  if (k1 <= k0) return cudaSuccess;
+  const uint32_t cpf = uint32_t(cdiv(F, kRleChunk));
+  uint64_t slots, cap, off_cnt, off_pc, bytes;
+  rle_dtmp_layout(n, F, k0, k1, &slots, &cap, &off_cnt, &off_pc, &bytes);
   uint64_t* cs = reinterpret_cast<uint64_t*>(tmp);
   uint32_t* cnt = reinterpret_cast<uint32_t*>(tmp + off_cnt);
   RlePiece* pcs = reinterpret_cast<RlePiece*>(tmp + off_pc);
@@ -413,9 +429,7 @@ cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int 
                                                           pcs, cnt, cap, sc, err);
     rle_fill_kernel<uint16_t><<<fgrid, kThreads, 0, st>>>(static_cast<uint16_t*>(out), pcs, cnt);
   }
-  e = cudaGetLastError();
-  cudaFreeAsync(tmp, st);
-  return e;
+  return cudaGetLastError();
 }
 
 }  // namespace cswap

@@ -102,6 +102,7 @@ _SIGS = {
     "cswap_status_string": (ctypes.c_char_p, [_i]),
     "cswap_last_error": (ctypes.c_char_p, []),
     "cswap_kernel_launches": (_u64, []),
+    "cswap_graph_stats": (None, [_P(_u64), _P(_u64)]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_L, _name)
@@ -306,6 +307,13 @@ def collect_kernel_timing(cap: int = 1 << 16):
 
 def kernel_launches() -> int:
     return int(_L.cswap_kernel_launches())
+
+
+def graph_stats() -> tuple[int, int]:
+    """(graph launches, graph instantiations) since init."""
+    a, b = _u64(0), _u64(0)
+    _L.cswap_graph_stats(ctypes.byref(a), ctypes.byref(b))
+    return int(a.value), int(b.value)
 
 
 def status_string(s: int) -> str:

@@ -1,0 +1,91 @@
+"""Launch groups replayed as CUDA graphs (api.cu run_group): the graph path is the
+one that runs, a cached executable graph updated in place for a differently sized / shaped
+call still produces the oracle's bytes, and the plain-launch path (CSWAP_GRAPHS=0, in a
+subprocess) gives the same containers."""
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import oracle as O
+from tests import gpu_util as G
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def C():
+    return G.lib()
+
+
+def test_swap_uses_graphs(C):
+    import torch
+    n = (1 << 21) + 77
+    x = synth.relu_iid(n, 0.5, seed=3)
+    d = G.to_dev(x)
+    g0, _ = C.graph_stats()
+    h = C.swap_out(d, n, C.F32, C.ZVC)
+    out = G.empty_like_words(n, 0)
+    h.swap_in(out)
+    h.wait()
+    torch.cuda.synchronize()
+    g1, _ = C.graph_stats()
+    assert g1 - g0 >= 2, "compress and decode groups should each be one graph launch"
+    assert np.array_equal(G.from_dev(out)[:n], x)
+    h.close()
+
+
+@pytest.mark.parametrize("codec", [1, 2, 3, 4])
+def test_graph_reuse_across_sizes(C, codec):
+    """The same (stream, group) executable graph is updated with new pointers, sizes and grid
+    shapes on every call: alternate sizes that change the frame count and the tail."""
+    import torch
+    C.set_format(1 << 20, 1024, 65536)
+    try:
+        for i, n in enumerate([5000, (1 << 20) * 3 + 17, 1 << 20, 33, (1 << 21) + 1024, 5000]):
+            for dt in (0, 1):
+                x = synth.relu_clustered(n, 0.6, 32, seed=100 + i, dtype=dt) if codec == 4 else \
+                    synth.relu_iid(n, 0.6, seed=100 + i, dtype=dt)
+                ref = O.compress(x, codec, dt, F=1 << 20, param={3: 1024, 4: 65536}.get(codec, 0))
+                assert G.gpu_compress(C, x, codec, dt, fmt=(1 << 20, 1024, 65536)) == ref, (n, dt)
+                y, err = G.gpu_decompress(C, ref, n, dt, codec, fmt=(1 << 20, 1024, 65536))
+                assert err == 0 and np.array_equal(y, x), (n, dt)
+                d = G.to_dev(x)
+                h = C.swap_out(d, n, dt, codec)
+                h.wait()
+                assert h.host_bytes() == ref
+                out = G.empty_like_words(n, dt)
+                h.swap_in(out)
+                h.wait()
+                torch.cuda.synchronize()
+                assert np.array_equal(G.from_dev(out)[:n], x)
+                h.close()
+    finally:
+        C.set_format(1 << 22, 1024, 65536)
+
+
+def test_plain_launch_path_matches():
+    """CSWAP_GRAPHS=0: same containers through plainly launched kernels (fresh process)."""
+    code = (
+        "import numpy as np, torch, synth\n"
+        "from oracle import oracle as O\n"
+        "from tests import gpu_util as G\n"
+        "C = G.lib()\n"
+        "for codec in (1, 2, 3, 4):\n"
+        "    n = (1 << 22) + 999\n"
+        "    x = synth.relu_iid(n, 0.7, seed=codec)\n"
+        "    d = G.to_dev(x)\n"
+        "    h = C.swap_out(d, n, 0, codec); h.wait()\n"
+        "    assert h.host_bytes() == O.compress(x, codec, 0), codec\n"
+        "    out = G.empty_like_words(n, 0); h.swap_in(out); h.wait(); torch.cuda.synchronize()\n"
+        "    assert np.array_equal(G.from_dev(out)[:n], x), codec\n"
+        "    h.close()\n"
+        "assert C.graph_stats()[0] == 0\n"
+        "print('plain ok')\n")
+    env = dict(os.environ, CSWAP_GRAPHS="0")
+    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and "plain ok" in r.stdout, r.stderr[-3000:]
