@@ -496,6 +496,17 @@ __global__ void __launch_bounds__(kThreads) zvc_count_kernel(const uint8_t* __re
   }
   const uint32_t* bm = reinterpret_cast<const uint32_t*>(in + fstart) + uint64_t(j) * G::WT;
   uint32_t c = 0;
+  if (tile_elems == uint32_t(G::TILE)) {  // full tile: all 16-byte loads issued back to back
+    constexpr int V = G::WT / 128;        // uint4 per lane (2 for f32, 4 for 16-bit)
+    uint4 v[V];
+#pragma unroll
+    for (int i = 0; i < V; i++) v[i] = __ldg(reinterpret_cast<const uint4*>(bm) + i * 32 + lane);
+#pragma unroll
+    for (int i = 0; i < V; i++) c += __popc(v[i].x) + __popc(v[i].y) + __popc(v[i].z) + __popc(v[i].w);
+    c = __reduce_add_sync(0xffffffffu, c);
+    if (lane == 0) sc.tbuf[t] = c;
+    return;
+  }
   for (uint32_t w = lane; w < nw; w += 32) {
     uint32_t x = bm[w];
     if (w == nw - 1 && (tile_elems & 31)) {
@@ -558,6 +569,7 @@ __global__ void __launch_bounds__(kThreads) zvc_expand_kernel(const uint8_t* __r
   using G = ZvcGeom<T>;
   __shared__ __align__(8) uint64_t s_bar;
   __shared__ __align__(16) uint32_t s_bm[G::WT + 4];
+  __shared__ uint32_t s_pre[G::WT];  // full tiles: non-zeros of the tile before bitmap word i
   __shared__ uint32_t s_woff[kWarps];
   extern __shared__ __align__(16) uint8_t s_val[];  // kTileBytes + 32
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -588,7 +600,72 @@ __global__ void __launch_bounds__(kThreads) zvc_expand_kernel(const uint8_t* __r
   }
   __syncthreads();
   mbar_wait(&s_bar, 0);
-  // per-warp totals
+  T* dst = outp + uint64_t(k) * F + uint64_t(j) * G::TILE;
+  if (tile_elems == uint32_t(G::TILE)) {
+    // ---- full tile (every tile but a frame's last): per-word exclusive prefix table, then per
+    // lane one bitmap word + one prefix load per 16-byte output vector (no per-word loops)
+    constexpr int WPT = G::WT / kThreads;  // bitmap words per thread for the table (1 or 2)
+    static_assert(WPT >= 1 && WPT * kThreads == G::WT, "expand geometry");
+    uint32_t pc[WPT], c = 0;
+#pragma unroll
+    for (int i = 0; i < WPT; i++) {
+      pc[i] = __popc(s_bm[tid * WPT + i]);
+      c += pc[i];
+    }
+    uint32_t inc = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += y;
+    }
+    if (lane == 31) s_woff[warp] = inc;
+    __syncthreads();
+    uint32_t base = 0, nnz = 0;
+#pragma unroll
+    for (int w = 0; w < kWarps; w++) {
+      const uint32_t x = s_woff[w];
+      base += w < warp ? x : 0;
+      nnz += x;
+    }
+    uint32_t run = base + inc - c;
+#pragma unroll
+    for (int i = 0; i < WPT; i++) {
+      s_pre[tid * WPT + i] = run;
+      run += pc[i];
+    }
+    __syncthreads();
+    const uint64_t vlast = vbeg + uint64_t(nnz) * G::W;
+    const bool ok = span_ok && (vend ? vend == vlast : a16(vlast) <= fend);
+    if (!ok && tid == 0) set_error(err, kErrCorrupt);
+    const uint32_t sv = uint32_t(__cvta_generic_to_shared(s_val)) + d;  // shared address of value 0
+#pragma unroll 2
+    for (int q = 0; q < G::NCH; q++) {
+      const uint32_t e0 = warp * G::PER_WARP + q * G::CHUNK + lane * G::EPV;
+      const uint32_t wi = e0 >> 5, sh = e0 & 31;
+      const uint32_t mine = s_bm[wi];
+      uint32_t a = sv + G::W * (s_pre[wi] + __popc(mine & ((1u << sh) - 1u)));
+      const uint32_t b = mine >> sh;
+      uint32_t w4[4];
+#pragma unroll
+      for (int e = 0; e < G::EPV; e++) {
+        const bool on = (b >> e) & 1u;
+        uint32_t x = 0;
+        if constexpr (sizeof(T) == 4) {
+          if (on) x = lds_u32(a);
+          w4[e] = x;
+        } else {
+          if (on) x = lds_u16(a);
+          if (e & 1) w4[e >> 1] |= x << 16;
+          else w4[e >> 1] = x;
+        }
+        a += on ? G::W : 0;
+      }
+      if (!ok) w4[0] = w4[1] = w4[2] = w4[3] = 0;
+      stg_stream(reinterpret_cast<uint4*>(dst + e0), make_uint4(w4[0], w4[1], w4[2], w4[3]));
+    }
+    return;
+  }
+  // ---- a frame's short last tile: bounds-checked general path
   {
     constexpr int WPW = G::WT / kWarps;
     uint32_t c = 0;
@@ -612,9 +689,8 @@ __global__ void __launch_bounds__(kThreads) zvc_expand_kernel(const uint8_t* __r
   const uint64_t vlast = vbeg + uint64_t(nnz) * G::W;
   const bool ok = span_ok && (vend ? vend == vlast : a16(vlast) <= fend);
   if (!ok && tid == 0) set_error(err, kErrCorrupt);
-  T* dst = outp + uint64_t(k) * F + uint64_t(j) * G::TILE;
   uint32_t r = woff;
-#pragma unroll
+#pragma unroll 1
   for (int q = 0; q < G::NCH; q++) {
     const uint32_t e0 = warp * G::PER_WARP + q * G::CHUNK + lane * G::EPV;
     const uint32_t cw0 = (warp * G::PER_WARP + q * G::CHUNK) / 32;
