@@ -185,6 +185,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
         assert torch.equal(o, t), "swap round trip mismatch"
 
     roof = _roofline(main["records"], args.steps)
+    roof["isolated"] = _isolated(C, torch, tensors, sizes, dtype, w, [q["codec"] for q in main["handles"]], stream,
+                                 roof.get("peak"))
     result = {
         "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4), "higher_is_better": True, "scaling": "weak",
@@ -301,6 +303,49 @@ def _roofline(records, steps: int = 1) -> dict:
     out["all_kernels"] = {f"{names[c]}_{'c' if dd == 0 else 'dc'}": {
         "GBps": round(v["bytes"] / (v["ms"] * 1e-3) / 1e9, 1), "frac": round(v["bytes"] / (v["ms"] * 1e-3) / 1e9 / peak, 4),
         "ms_total": round(v["ms"], 3), "launches": v["launches"]} for (c, dd), v in groups.items()}
+    return out
+
+
+def _isolated(C, torch, tensors, sizes, dtype, w, codecs, stream, peak, reps=3) -> dict:
+    """The same codec launches with no copy engine running: each tensor of the set compressed
+    (device -> device) and decompressed with its chosen codec, CUDA events around every call.
+    In the timed step every launch group shares the GPU with a D2H / H2D copy, and then each
+    event record and kernel boundary waits ~10-20 us behind the copy's queued PCIe writes
+    (tools/launch_probe*.py); this shows what the kernels reach without that."""
+    out = {}
+    work = [(t, n, c) for t, n, c in zip(tensors, sizes, codecs) if c != C.NONE]
+    if not work:
+        return out
+    cap = max(C.max_compressed_size(n, dtype, c) for _, n, c in work)
+    buf = torch.empty(cap, dtype=torch.uint8, device="cuda")
+    size = torch.zeros(1, dtype=torch.int64, device="cuda")
+    dst = torch.empty(max(n for _, n, _ in work) * w, dtype=torch.uint8, device="cuda")
+    err = torch.zeros(1, dtype=torch.int32, device="cuda")
+    tc = td = 0.0
+    nbytes = 0
+    for t, n, c in work:
+        for r in range(reps + 1):
+            a, b, d = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+            # keep the stream busy while the host enqueues, so that the events time the device
+            # work and not the host-side capture of the launch group
+            torch.cuda._sleep(100000)
+            a.record(stream)
+            C.compress(t, n, dtype, c, buf, cap, size, stream=stream)
+            b.record(stream)
+            C.decompress(buf, cap, dst, n, dtype, c, err=err, stream=stream)
+            d.record(stream)
+            d.synchronize()
+            if r:  # the first round is a warm-up
+                tc += a.elapsed_time(b)
+                td += b.elapsed_time(d)
+                nbytes += n * w + int(size.item())
+    assert int(err.item()) == 0
+    for name, ms in (("compress", tc), ("decompress", td)):
+        gbs = nbytes / (ms * 1e-3) / 1e9
+        out[name] = {"achieved": round(gbs, 1), "frac": round(gbs / peak, 4) if peak else None,
+                     "avg_launch_ms": round(ms / (reps * len(work)), 4)}
+    out["how"] = (f"every tensor of the set with its chosen codec, device->device, no copy running, "
+                  f"{reps} reps after a warm-up, CUDA events per call on the launching stream")
     return out
 
 

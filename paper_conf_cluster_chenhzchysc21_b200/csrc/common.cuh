@@ -18,6 +18,7 @@ enum : uint32_t { kErrOK = 0, kErrCorrupt = 5 };
 
 __host__ __device__ __forceinline__ uint64_t a16(uint64_t x) { return (x + 15) & ~uint64_t(15); }
 __host__ __device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__host__ __device__ __forceinline__ uint32_t umin32(uint32_t a, uint32_t b) { return a < b ? a : b; }
 __host__ __device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a > b ? a : b; }
 __host__ __device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 __host__ __device__ __forceinline__ uint64_t data_start(uint32_t K) { return a16(64 + 8ull * K); }
@@ -235,6 +236,30 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
       : "memory");
 }
 
+// Wait with exponential __nanosleep backoff (32 ns .. max_ns) between non-blocking phase tests:
+// for warps whose wait is off the critical path (a polling warp issues an instruction every ~20
+// cycles even with try_wait's suspend hint, taking issue slots from the warps that do the work)
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t phase) {
+  uint32_t a = static_cast<uint32_t>(__cvta_generic_to_shared(bar)), ok;
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      "selp.u32 %0, 1, 0, p;\n"
+      "}\n"
+      : "=r"(ok)
+      : "r"(a), "r"(phase)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t phase, uint32_t max_ns) {
+  uint32_t ns = 32;
+  while (!mbar_test(bar, phase)) {
+    __nanosleep(ns);
+    ns = ns < max_ns ? ns * 2 : max_ns;
+  }
+}
+
 // ---- vector helpers -------------------------------------------------------------------
 __device__ __forceinline__ uint4 ldg_stream(const uint4* p) {
   uint4 r;
@@ -252,6 +277,11 @@ __device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
 __device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
   uint16_t v;
   asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ uint4 lds_v4(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
   return v;
 }
 __device__ __forceinline__ void stg_stream(uint4* p, uint4 v) {

@@ -109,6 +109,14 @@ constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 #define CSWAP_ZVC_MAX_BACKOFF 32
 #endif
 constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
+// mbarrier waits sleep between tests (max ns): the producer refills a stage whose TMA load takes
+// ~1 us anyway; a resolver has LAG tile periods (~1.5 us each) before its offset is needed; the
+// polling consumer warp is on the critical path and sleeps least
+#ifndef CSWAP_ZVC_SLEEP
+#define CSWAP_ZVC_SLEEP 1
+#endif
+constexpr uint32_t kProducerSleep = 256 * CSWAP_ZVC_SLEEP, kResolverSleep = 128 * CSWAP_ZVC_SLEEP,
+                   kConsumerSleep = 64 * CSWAP_ZVC_SLEEP;
 
 #ifndef CSWAP_ZVC_DYNAMIC_TILES
 constexpr bool kStaticTiles = true;
@@ -193,7 +201,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     for (uint32_t i = 0;; i++) {
       const int s = i % S;
       long long c0 = clock64();
-      if (i >= S) mbar_wait(&bar_empty[s], ((i / S) - 1) & 1);
+      if (i >= S) mbar_wait_sleep(&bar_empty[s], ((i / S) - 1) & 1, kProducerSleep);
       if (lane == 0) ZPROF_ADD(0, clock64() - c0);
       // static round-robin assignment: CTA b takes tiles b, b + G, b + 2G, ... so every CTA
       // counts the tiles of round r at about the same time and a tile's offset waits only for
@@ -229,7 +237,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     for (uint32_t i = r;; i += S) {
       const int s = r;
       long long c0 = clock64();
-      mbar_wait(&bar_cnt[s], (i / S) & 1);
+      mbar_wait_sleep(&bar_cnt[s], (i / S) & 1, kResolverSleep);
       long long c1 = clock64();
       if (lane == 0) ZPROF_ADD(2, c1 - c0);
       const uint32_t nnz = s_nnz[s];
@@ -334,7 +342,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
   };
   constexpr int EROWS = PW / 32;  // rows of 32 elements per slab
   auto group_wait = [&](uint64_t* bar, uint32_t parity) {  // one warp polls, the rest block in bar.sync
-    if (warp == 0) mbar_wait(bar, parity);
+    if (warp == 0) mbar_wait_sleep(bar, parity, kConsumerSleep);
     consumer_sync();
     if (warp != 0) mbar_wait(bar, parity);  // phase already complete: returns at once
   };
@@ -366,13 +374,36 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     return tot;
   };
 
-  // copy the slab's compacted non-zeros (count_slab) to the container: full-warp stores of
-  // consecutive words
+  // copy the slab's compacted non-zeros (count_slab) to the container: element stores up to the
+  // destination's next 16-byte boundary, then 16-byte stores whose source is the smem slab
+  // funnel-shifted by that head (k whole words + r bits, warp-uniform), then the element tail
   auto emit_slab = [&](const uint8_t* stage, uint32_t cnt, uint8_t* dst) {
     const T* sv = reinterpret_cast<const T*>(stage) + warp * PW;
     T* d = reinterpret_cast<T*>(dst);
-#pragma unroll 4
-    for (uint32_t q = lane; q < cnt; q += 32) d[q] = sv[q];
+    const uint32_t nbytes = cnt * G::W;
+    const uint32_t h = umin32((16u - (uint32_t(reinterpret_cast<uintptr_t>(dst)) & 15u)) & 15u, nbytes);
+    const uint32_t nb = (nbytes - h) >> 4, tail = h + 16 * nb;
+    if (uint32_t(lane) < h / G::W) d[lane] = sv[lane];
+    if (uint32_t(lane) < (nbytes - tail) / G::W) d[tail / G::W + lane] = sv[tail / G::W + lane];
+    const uint32_t sa = uint32_t(__cvta_generic_to_shared(sv));
+    uint4* dv = reinterpret_cast<uint4*>(dst + h);
+    auto body = [&](auto kk) {
+      constexpr int k = decltype(kk)::value;
+      const uint32_t r = (h & 3u) * 8u;
+#pragma unroll 2
+      for (uint32_t q = lane; q < nb; q += 32) {
+        const uint4 A = lds_v4(sa + 16 * q), B = lds_v4(sa + 16 * q + 16);
+        const uint32_t w[8] = {A.x, A.y, A.z, A.w, B.x, B.y, B.z, B.w};
+        stg_stream(dv + q, make_uint4(__funnelshift_r(w[k], w[k + 1], r), __funnelshift_r(w[k + 1], w[k + 2], r),
+                                      __funnelshift_r(w[k + 2], w[k + 3], r), __funnelshift_r(w[k + 3], w[k + 4], r)));
+      }
+    };
+    switch (h >> 2) {
+      case 0: body(std::integral_constant<int, 0>{}); break;
+      case 1: body(std::integral_constant<int, 1>{}); break;
+      case 2: body(std::integral_constant<int, 2>{}); break;
+      default: body(std::integral_constant<int, 3>{}); break;
+    }
   };
 
   auto count = [&](uint32_t i, uint32_t t) {
