@@ -104,7 +104,7 @@ class SwapSaver:
     """
 
     def __init__(self, policy="auto", min_bytes: int = 1 << 20, prefetch: bool = True, backend=None,
-                 verify: bool = False):
+                 verify: bool = False, reprofile_every: int = 0):
         if not (isinstance(policy, int) or policy in ("resident", *POLICIES)):
             raise ValueError(f"unknown policy {policy!r}")
         self.policy = policy
@@ -114,6 +114,14 @@ class SwapSaver:
         self.verify = verify  # debug: keep a device copy of every swapped tensor, compare on use
         self.mismatches: list[tuple[int, int]] = []
         self.hidden: list[tuple[float, float]] | None = None
+        # online re-profiling (NEXT-2; PAPER.md:118 "sparsity ... per epoch", :156-162): with
+        # reprofile_every = N > 0 the AUTO policy probes and decides only on every N-th step
+        # (a profiling step) and replays the stored execution plan — one codec per tensor index —
+        # on the others, which then skip the probe and its host synchronisation
+        self.reprofile_every = reprofile_every
+        self.step_index = -1
+        self.plan: list[int] | None = None
+        self.plan_history: list[tuple[int, list[int]]] = []
         self._order: list[_Rec] = []
         self._live: dict = {}
         self._ctx = None
@@ -140,6 +148,9 @@ class SwapSaver:
             self.backend = CSwapBackend()
         self._order, self._live = [], {}
         self.stats = {"swapped": 0, "raw_bytes": 0, "comp_bytes": 0, "codecs": []}
+        self.step_index += 1
+        self._profiling = (self.policy == "auto" and (self.reprofile_every <= 0 or self.plan is None
+                                                      or self.step_index % self.reprofile_every == 0))
         self._ctx = torch.autograd.graph.saved_tensors_hooks(self._pack, self._unpack)
         self._ctx.__enter__()
         return self
@@ -147,6 +158,9 @@ class SwapSaver:
     def __exit__(self, *exc):
         self._ctx.__exit__(*exc)
         self._ctx = None
+        if self.policy == "auto" and self.reprofile_every > 0 and self._profiling:
+            self.plan = list(self.stats["codecs"])
+            self.plan_history.append((self.step_index, self.plan))
         return False
 
     def _pack(self, t):
@@ -165,6 +179,8 @@ class SwapSaver:
         i = len(self._order)
         hf, hb = self.hidden[i] if self.hidden and i < len(self.hidden) else (0.0, 0.0)
         codec = self.policy if isinstance(self.policy, int) else POLICIES[self.policy]
+        if codec == C.AUTO and not self._profiling and self.plan is not None and i < len(self.plan):
+            codec = self.plan[i]
         rec = _Rec(i, t.shape, t.dtype, t.device, t.numel() * t.element_size())
         rec.ref = weakref.ref(t)
         if self.verify:

@@ -136,3 +136,42 @@ def test_reused_address_is_not_deduplicated():
     assert all(torch.equal(a, b) for a, b in zip(got, ref))
     # x and the 8 relu outputs: each its own record, however the allocator reused addresses
     assert saver.stats["swapped"] == len(be.out) == 9
+
+
+class Deciding(HostCopy):
+    """AUTO stand-in: 'compresses' (codec 1) iff the tensor has any zero, else NONE."""
+
+    def swap_out(self, t, codec, hf, hb):
+        h = super().swap_out(t, codec, hf, hb)
+        self.decided = getattr(self, "decided", 0) + (codec == 255)
+        return (h, 1 if codec == 1 or (codec == 255 and bool((t == 0).any())) else 0)
+
+    def swap_in(self, h, out, stream):
+        super().swap_in(h[0], out, stream)
+
+    @staticmethod
+    def info(h):
+        return h[1], h[0].numel() * h[0].element_size()
+
+
+def test_reprofiling_replays_plan_between_profiling_steps():
+    be = Deciding()
+    saver = SwapSaver(policy="auto", min_bytes=0, backend=be, reprofile_every=3)
+    w = torch.randn(64, 64, requires_grad=True)
+    shift = 1000.0  # large positive bias: no zeros -> NONE
+    plans = []
+    for step in range(7):
+        if step == 3:
+            shift = -1000.0  # drift: every relu output becomes all zero -> compress
+        x = torch.randn(32, 64)
+        with saver:
+            y = torch.relu(x @ w + shift)
+            loss = (y * y).sum()
+        loss.backward()
+        plans.append(list(saver.stats["codecs"]))
+    # steps 0, 3, 6 are profiling steps (AUTO asked per tensor); the others replay the plan
+    assert [s for s, _ in saver.plan_history] == [0, 3, 6]
+    # saved: x (the matmul input, never zero) and the relu output y
+    assert plans[0] == plans[1] == plans[2] == [0, 0]
+    assert plans[3] == plans[4] == plans[5] == [0, 1]
+    assert be.decided == sum(len(plans[i]) for i in (0, 3, 6))
