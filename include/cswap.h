@@ -109,6 +109,14 @@ cswap_status cswap_get_calibration(cswap_calib* out);
 /* Default format used by cswap_swap_out and by calls passing fmt = NULL. */
 cswap_status cswap_set_format(const cswap_format* fmt);
 cswap_status cswap_get_format(cswap_format* out);
+/* Launch configuration of the persistent ZVC compress kernel (the knob PAPER.md §IV-D / Alg. 1,
+ * :170-214, tunes by Bayesian optimisation on V100: grid x block).  grid = CTAs (0 = automatic:
+ * SM count x resident CTAs per SM; clamped to that co-resident maximum, which the kernel's
+ * cross-CTA offset protocol needs for forward progress); variant = stage/tile geometry
+ * (0: 3 x 32 KiB stages, 1: 6 x 16 KiB, 2: 5 x 16 KiB, 3: 4 x 16 KiB; -1 = default / the
+ * CSWAP_ZVC_CFG environment variable).  Process-wide; returns CSWAP_ERR_INVALID for a variant
+ * outside -1..3. */
+cswap_status cswap_set_zvc_launch(uint32_t grid, int32_t variant);
 
 /* ---- device codecs (a3-a10) ------------------------------------------------------------------ */
 /* Worst-case container bytes for n elements (0 on invalid arguments).  fmt may be NULL. */

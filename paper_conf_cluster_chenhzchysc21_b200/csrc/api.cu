@@ -733,6 +733,11 @@ cswap_status cswap_set_format(const cswap_format* f) {
   return CSWAP_OK;
 }
 
+cswap_status cswap_set_zvc_launch(uint32_t grid, int32_t variant) {
+  if (!zvc_set_launch(grid, variant)) return fail(CSWAP_ERR_INVALID, "variant %d outside -1..3", int(variant));
+  return CSWAP_OK;
+}
+
 cswap_status cswap_get_format(cswap_format* out) {
   if (!out) return fail(CSWAP_ERR_INVALID, "out is NULL");
   *out = g_ctx ? g_ctx->fmt : cswap_format{uint64_t(1) << 22, 1024, 65536};

@@ -32,6 +32,7 @@ cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, c
 // zvc.cu
 uint32_t zvc_tiles(uint64_t n, int w, uint64_t F, uint32_t k0, uint32_t k1, uint32_t* tpf_out);
 void zvc_compress_scratch(uint64_t n, int w, uint64_t F, uint64_t* tiles, uint64_t* aux);
+bool zvc_set_launch(uint32_t grid, int variant);  // cswap_set_zvc_launch
 cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
                                 const Scratch& sc, uint32_t epoch, int dtype, cudaStream_t st);
 cudaError_t launch_zvc_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, uint32_t k0,

@@ -18,6 +18,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <atomic>
 #include <type_traits>
 
 #include "common.cuh"
@@ -775,6 +776,9 @@ uint32_t zvc_tiles(uint64_t n, int w, uint64_t F, uint32_t k0, uint32_t k1, uint
   return (k1 - 1 - k0) * tpf + uint32_t(cdiv(frame_len(n, F, k1 - 1), TILE));
 }
 
+static std::atomic<uint32_t> g_zvc_grid{0};
+static std::atomic<int> g_zvc_variant{-1};
+
 static int prof_enabled() {
   static int p = -1;
   if (p < 0) p = getenv("CSWAP_ZVC_PROF") ? 1 : 0;
@@ -807,7 +811,9 @@ static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uin
   const uint32_t per_sm = L::ctas_per_sm;
   // per-frame and per-group (tiles, nnz) accumulators
   launch_zero_words(sc.aux2, (uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32)) * 2, st);
-  const uint32_t grid = std::min<uint32_t>(tiles, uint32_t(sm_count()) * per_sm);
+  const uint32_t cap = uint32_t(sm_count()) * per_sm;  // co-resident maximum (forward progress)
+  const uint32_t want = g_zvc_grid.load(std::memory_order_relaxed);
+  const uint32_t grid = std::min<uint32_t>(tiles, want ? std::min(want, cap) : cap);
   timing_kernel_start(st);
   zvc_compress_persistent<T, S, CW, TB><<<grid, compress_threads<S, CW>(), L::bytes, st>>>(
       static_cast<const T*>(in), n, F, K, tpf, tiles, out, out_size, sc, epoch, dtype, prof_enabled());
@@ -827,8 +833,10 @@ static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uin
   return cudaGetLastError();
 }
 
-// compress configuration (stages x consumer warps); CSWAP_ZVC_CFG overrides for experiments
+// compress configuration (stages x tile bytes): cswap_set_zvc_launch, else CSWAP_ZVC_CFG, else 0
 static int compress_cfg() {
+  const int v = g_zvc_variant.load(std::memory_order_relaxed);
+  if (v >= 0) return v;
   static int c = -1;
   if (c < 0) {
     const char* e = getenv("CSWAP_ZVC_CFG");
@@ -836,6 +844,13 @@ static int compress_cfg() {
     if (c < 0 || c > 3) c = 0;
   }
   return c;
+}
+
+bool zvc_set_launch(uint32_t grid, int variant) {
+  if (variant < -1 || variant > 3) return false;
+  g_zvc_grid.store(grid);
+  g_zvc_variant.store(variant);
+  return true;
 }
 
 template <typename T>

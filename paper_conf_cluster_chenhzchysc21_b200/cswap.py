@@ -103,6 +103,7 @@ _SIGS = {
     "cswap_last_error": (ctypes.c_char_p, []),
     "cswap_kernel_launches": (_u64, []),
     "cswap_graph_stats": (None, [_P(_u64), _P(_u64)]),
+    "cswap_set_zvc_launch": (_i, [_u32, ctypes.c_int32]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_L, _name)
@@ -307,6 +308,11 @@ def collect_kernel_timing(cap: int = 1 << 16):
 
 def kernel_launches() -> int:
     return int(_L.cswap_kernel_launches())
+
+
+def set_zvc_launch(grid: int = 0, variant: int = -1):
+    """Persistent ZVC compress launch: grid CTAs (0 = auto) and stage/tile variant (-1 = default)."""
+    _check(_L.cswap_set_zvc_launch(grid, variant), "cswap_set_zvc_launch")
 
 
 def graph_stats() -> tuple[int, int]:
