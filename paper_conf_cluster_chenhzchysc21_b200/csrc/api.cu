@@ -392,10 +392,18 @@ struct Lease {
   cswap_status status = CSWAP_OK;
   Lease(Ctx& c, cudaStream_t s, uint64_t tiles, uint64_t aux) : ctx(&c), st(s) {
     const uint32_t start = c.rr.fetch_add(1);
-    for (int i = 0; i < kBlocks && !b; i++) {
-      Block& cand = c.blocks[(start + i) % kBlocks];
-      std::unique_lock<std::mutex> l(cand.m, std::try_to_lock);
-      if (l.owns_lock()) {
+    // prefer a free block that is already large enough: growing one (ensure_block) frees and
+    // re-allocates device memory, which synchronises the device — if every block had to grow
+    // in turn, each of the first kBlocks large operations would pay that (a calibration sample
+    // measured 99 ms for a 256 MiB decode that way)
+    for (int pass = 0; pass < 2 && !b; pass++) {
+      for (int i = 0; i < kBlocks && !b; i++) {
+        Block& cand = c.blocks[(start + i) % kBlocks];
+        std::unique_lock<std::mutex> l(cand.m, std::try_to_lock);
+        if (!l.owns_lock()) continue;
+        if (pass == 0 && !(cand.sc.status && cand.sc.cap_tiles >= std::max<uint64_t>(tiles, 1024) &&
+                           cand.sc.cap_aux >= std::max<uint64_t>(aux, 1024)))
+          continue;
         b = &cand;
         lk = std::move(l);
       }
