@@ -40,7 +40,7 @@ def main():
     y = torch.randint(0, 1000, (a.batch,), device="cuda")
     init = {k: v.clone() for k, v in model.state_dict().items()}
 
-    after_fwd = []
+    after_fwd, fwd_peak = [], []
 
     def fwd_bwd(saver, mark=None):
         torch.manual_seed(1)  # same dropout masks in every run (bitwise gradient comparison)
@@ -53,6 +53,7 @@ def main():
         if mark:
             mark()
         after_fwd.append(torch.cuda.memory_allocated())
+        fwd_peak.append(torch.cuda.max_memory_allocated())
         loss.backward()
         return loss
 
@@ -78,6 +79,7 @@ def main():
         torch.cuda.synchronize()
         torch.cuda.reset_peak_memory_stats()
         after_fwd.clear()
+        fwd_peak.clear()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t0 = time.perf_counter()
         e0.record()
@@ -90,7 +92,8 @@ def main():
         ms = e0.elapsed_time(e1) / a.iters
         row = {"policy": pol, "ms_per_iter": round(ms, 2), "wall_ms_per_iter": round(wall, 2),
                "peak_GiB": round(torch.cuda.max_memory_allocated() / 2**30, 2),
-               "after_fwd_GiB": round(max(after_fwd) / 2**30, 2), "grads_bitwise_equal": exact}
+               "after_fwd_GiB": round(max(after_fwd) / 2**30, 2),
+               "fwd_peak_GiB": round(fwd_peak[0] / 2**30, 2), "grads_bitwise_equal": exact}
         if saver is not None:
             st = saver.stats
             row.update({"swapped_tensors": st["swapped"], "raw_MiB": round(st["raw_bytes"] / 2**20, 1),
