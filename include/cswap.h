@@ -185,11 +185,15 @@ cswap_status cswap_fit_linear(const double* X, const double* y, uint64_t m, uint
 /* ---- kernel timing (bench / profiling) --------------------------------------------------------- */
 /* One record per timed codec launch group: direction 0 = compress, 1 = decompress, 2 = probe;
  * raw_bytes = uncompressed bytes covered, comp_bytes = container bytes read or written (0 if
- * unknown), ms = CUDA-event time on the launch stream. */
+ * unknown), ms = CUDA-event time on the launch stream; device_ms = %globaltimer difference
+ * between two 1-thread stamp kernels placed first and last in the group's graph (the group's
+ * own device duration, without the event records' waits behind concurrent PCIe traffic;
+ * 0 if unavailable). */
 typedef struct {
   int32_t codec, direction;
   uint64_t raw_bytes, comp_bytes;
   double ms;
+  double device_ms;
 } cswap_kernel_record;
 /* When enabled, the swap pipeline brackets its probe / compress / decompress launches with CUDA
  * events on the stream they are launched on. */

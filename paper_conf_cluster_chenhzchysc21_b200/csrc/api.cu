@@ -176,6 +176,7 @@ struct Ctx {
   struct Pend {
     cudaEvent_t a, b;
     cswap_kernel_record r;
+    uint64_t* stamps;  // 2 x u64 %globaltimer (mapped pinned), or null
   };
   std::vector<Pend> pend;
 };
@@ -190,9 +191,8 @@ struct Timer {
   cudaStream_t st;
   cudaEvent_t a = nullptr, b = nullptr;
   bool started = false;
-  Timer(Ctx* ctx, cudaStream_t s) : c(ctx), st(s) {
-    if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) t_pending = this;
-  }
+  uint64_t* stamps = nullptr;  // filled by stamp kernels first / last in the group (run_group)
+  Timer(Ctx* ctx, cudaStream_t s);
   void start_now() {
     if (a && !started) {
       cudaEventRecord(a, st);
@@ -208,15 +208,28 @@ struct Timer {
     if (!a) return;
     stop();
     std::lock_guard<std::mutex> lk(c->tm_m);
-    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0}});
+    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0, 0.0}, stamps});
     a = b = nullptr;
+    stamps = nullptr;
   }
-  ~Timer() {
-    if (t_pending == this) t_pending = nullptr;
-    if (a) cudaEventDestroy(a);
-    if (b) cudaEventDestroy(b);
-  }
+  ~Timer();
 };
+}  // namespace
+
+namespace {
+Timer::Timer(Ctx* ctx, cudaStream_t s) : c(ctx), st(s) {
+  if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) {
+    t_pending = this;
+    stamps = reinterpret_cast<uint64_t*>(c->pinned.alloc(16));
+    if (stamps) stamps[0] = stamps[1] = 0;
+  }
+}
+Timer::~Timer() {
+  if (t_pending == this) t_pending = nullptr;
+  if (a) cudaEventDestroy(a);
+  if (b) cudaEventDestroy(b);
+  if (stamps) c->pinned.free(reinterpret_cast<uint8_t*>(stamps));  // not committed
+}
 }  // namespace
 
 void cswap::timing_kernel_start(cudaStream_t) {
@@ -237,6 +250,7 @@ namespace {
 // (thread, stream, group key) and updated in place (cudaGraphExecUpdate) with the new pointers /
 // sizes; it is re-instantiated only when the topology changes.  CSWAP_GRAPHS=0 launches plainly.
 std::atomic<uint64_t> g_gen{0};
+cswap_status cuda_status(cudaError_t e, const char* what);
 
 bool graphs_enabled() {
   static int on = -1;
@@ -274,16 +288,33 @@ constexpr size_t kGraphCacheMax = 64;
 // graph launch (timing events cannot be recorded inside a capture).
 template <class Fn>
 cswap_status run_group(Ctx* c, cudaStream_t st, uint64_t key, Fn&& fn) {
-  if (!graphs_enabled()) return fn(st);
+  Timer* pending = t_pending;
+  uint64_t* stamps = pending ? pending->stamps : nullptr;
+  // timed groups: stamp kernels first and last (device duration of the group)
+  auto body = [&](cudaStream_t gs) -> cswap_status {
+    if (stamps) {
+      c->launches++;
+      TRY(cuda_status(launch_stamp(stamps, gs), "stamp"));
+    }
+    TRY(fn(gs));
+    if (stamps) {
+      c->launches++;
+      TRY(cuda_status(launch_stamp(stamps + 1, gs), "stamp"));
+    }
+    return CSWAP_OK;
+  };
+  if (!graphs_enabled()) {
+    if (pending) pending->start_now();
+    return body(st);
+  }
   GraphCache& g = t_gc;
   if (g.gen != c->gen) g.reset(c->gen);
   if (!g.cap && cudaStreamCreateWithFlags(&g.cap, cudaStreamNonBlocking) != cudaSuccess)
     return fail(CSWAP_ERR_CUDA, "capture stream create failed");
   if (cudaStreamBeginCapture(g.cap, cudaStreamCaptureModeRelaxed) != cudaSuccess)
     return fail(CSWAP_ERR_CUDA, "begin capture failed: %s", cudaGetErrorString(cudaGetLastError()));
-  Timer* pending = t_pending;
   t_pending = nullptr;
-  cswap_status s = fn(g.cap);
+  cswap_status s = body(g.cap);
   t_pending = pending;
   cudaGraph_t graph = nullptr;
   const cudaError_t e = cudaStreamEndCapture(g.cap, &graph);
@@ -1172,6 +1203,11 @@ uint64_t cswap_collect_kernel_timing(cswap_kernel_record* out, uint64_t cap) {
     cudaEventSynchronize(e.b);
     cudaEventElapsedTime(&ms, e.a, e.b);
     e.r.ms = ms;
+    if (e.stamps) {  // written by the group's stamp kernels, complete once e.b is
+      const volatile uint64_t* t = e.stamps;
+      e.r.device_ms = (t[0] && t[1] > t[0]) ? double(t[1] - t[0]) * 1e-6 : 0.0;
+      c->pinned.free(reinterpret_cast<uint8_t*>(e.stamps));
+    }
     if (out && k < cap) out[k] = e.r;
     k++;
     cudaEventDestroy(e.a);

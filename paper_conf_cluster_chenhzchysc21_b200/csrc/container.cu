@@ -212,6 +212,18 @@ cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtyp
   return cudaGetLastError();
 }
 
+// ---- timing stamps: one thread writes %globaltimer (ns) --------------------------------------
+__global__ void stamp_kernel(unsigned long long* dst) {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  *dst = t;
+}
+
+cudaError_t launch_stamp(uint64_t* dst, cudaStream_t st) {
+  stamp_kernel<<<1, 1, 0, st>>>(reinterpret_cast<unsigned long long*>(dst));
+  return cudaGetLastError();
+}
+
 // ---- NONE decompress: frames are raw; check sizes, copy -----------------------------------
 __global__ void none_check_kernel(uint64_t n, uint64_t F, int w, const uint64_t* fbytes, uint32_t* err) {
   const uint32_t K = uint32_t(cdiv(n, F));
