@@ -60,13 +60,20 @@ def main():
         loss.backward()
 
     def timed(saver, n):
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
+        per = []
         for _ in range(n):
-            step(saver)
-        e1.record()
-        e1.synchronize()
-        return e0.elapsed_time(e1) / n
+            e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+            model.zero_grad(set_to_none=True)
+            e[0].record()
+            with saver:
+                loss = torch.nn.functional.cross_entropy(model(x), y)
+            e[1].record()
+            loss.backward()
+            e[2].record()
+            e[2].synchronize()
+            per.append((round(e[0].elapsed_time(e[1]), 2), round(e[1].elapsed_time(e[2]), 2)))
+        timed.last = per
+        return sum(a + b for a, b in per) / n
 
     relus = [m for m in model.features if isinstance(m, torch.nn.ReLU)]
     zf = []
@@ -93,7 +100,9 @@ def main():
         step(st)          # st: profiles once (epoch 0), then replays that plan
         step(st)
         ms_re = timed(re, a.steps)
+        per_re = timed.last
         ms_st = timed(st, a.steps)
+        per_st = timed.last
         plan = re.plan or []
         row = {"epoch": e, "target_sparsity": s, "relu_sparsity_mean": sp, "relu_all_zero": dead,
                "codecs_reprofiled": plan,
@@ -101,7 +110,8 @@ def main():
                "compressed_static": sum(1 for c in (st.plan or []) if c != 0), "tensors": len(plan),
                "ms_step_reprofiled": round(ms_re, 2), "ms_step_static": round(ms_st, 2),
                "host_MiB_reprofiled": round(re.stats["comp_bytes"] / 2**20, 1),
-               "host_MiB_static": round(st.stats["comp_bytes"] / 2**20, 1)}
+               "host_MiB_static": round(st.stats["comp_bytes"] / 2**20, 1),
+               "fwd_bwd_ms_reprofiled": per_re, "fwd_bwd_ms_static": per_st}
         rows.append(row)
         print(json.dumps(row), flush=True)
 
