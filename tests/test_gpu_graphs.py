@@ -89,3 +89,62 @@ def test_plain_launch_path_matches():
     env = dict(os.environ, CSWAP_GRAPHS="0")
     r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0 and "plain ok" in r.stdout, r.stderr[-3000:]
+
+
+@pytest.mark.parametrize("grid,variant", [(1, 0), (7, 1), (148, 2), (296, 3), (0, -1)])
+def test_zvc_launch_config_keeps_bytes(C, grid, variant):
+    """cswap_set_zvc_launch changes only how the persistent compress runs, never its bytes."""
+    n = (1 << 21) + 333
+    x = synth.relu_iid(n, 0.45, seed=11)
+    ref = O.compress(x, O.ZVC, O.F32)
+    try:
+        C.set_zvc_launch(grid, variant)
+        assert G.gpu_compress(C, x, O.ZVC, O.F32) == ref
+    finally:
+        C.set_zvc_launch(0, -1)
+
+
+def test_zvc_launch_config_rejects_bad_variant(C):
+    with pytest.raises(C.CswapError):
+        C.set_zvc_launch(0, 4)
+
+
+def test_timing_records_carry_device_clock(C):
+    """Timed launch groups carry a device-clock duration (stamp kernels) next to the event time."""
+    import torch
+    n = 8 << 20
+    x = synth.relu_iid(n, 0.5, seed=5)
+    d = G.to_dev(x)
+    out = G.empty_like_words(n, 0)
+    C.collect_kernel_timing()
+    C.set_kernel_timing(True)
+    try:
+        h = C.swap_out(d, n, C.F32, C.ZVC)
+        h.swap_in(out)
+        h.wait()
+        torch.cuda.synchronize()
+    finally:
+        C.set_kernel_timing(False)
+    recs = [r for r in C.collect_kernel_timing() if r["direction"] in (0, 1)]
+    assert recs and all(0 < r["device_ms"] <= r["ms"] * 1.05 + 0.01 for r in recs), recs
+    assert np.array_equal(G.from_dev(out)[:n], x)
+    h.close()
+
+
+def test_many_streams_evict_graph_cache(C):
+    """More (stream, group) pairs than the executable-graph cache holds: evicted graphs must not
+    disturb later launches."""
+    import torch
+    n = 100_000
+    x = synth.relu_iid(n, 0.5, seed=9)
+    ref = O.compress(x, O.ZVC, O.F32)
+    d = G.to_dev(x)
+    cap = C.max_compressed_size(n, C.F32, C.ZVC)
+    size = torch.zeros(1, dtype=torch.int64, device="cuda")
+    for i in range(80):
+        s = torch.cuda.Stream()
+        out = torch.zeros(cap, dtype=torch.uint8, device="cuda")
+        s.wait_stream(torch.cuda.current_stream())
+        C.compress(d, n, C.F32, C.ZVC, out, cap, size, stream=s)
+        s.synchronize()
+        assert out[: int(size.item())].cpu().numpy().tobytes() == ref, i
