@@ -46,42 +46,9 @@ struct ZvcGeom {
   static_assert(NCH * CHUNK * kWarps == TILE, "tile geometry");
 };
 
-template <typename T>
-__device__ __forceinline__ uint32_t nonzero_bits(uint4 v) {
-  if constexpr (sizeof(T) == 4) {
-    return (v.x != 0) | ((v.y != 0) << 1) | ((v.z != 0) << 2) | ((v.w != 0) << 3);
-  } else {
-    auto h = [](uint32_t u) { return ((u & 0xFFFFu) != 0) | (((u >> 16) != 0) << 1); };
-    return h(v.x) | (h(v.y) << 2) | (h(v.z) << 4) | (h(v.w) << 6);
-  }
-}
-template <typename T>
-__device__ __forceinline__ uint32_t lane_elem(const uint4& v, int i) {
-  const uint32_t w[4] = {v.x, v.y, v.z, v.w};
-  if constexpr (sizeof(T) == 4) return w[i];
-  else return (w[i >> 1] >> ((i & 1) * 16)) & 0xFFFFu;
-}
-
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(bar)))
                : "memory");
-}
-
-// Read EPV elements starting at tile-relative element e0: from the smem stage where the bulk copy
-// landed, from global memory for the sub-16-byte tail of the tensor, zero past the tile end.
-template <typename T>
-__device__ __forceinline__ uint4 tile_vec(const uint8_t* stage, const T* gsrc, uint32_t e0, uint32_t bulk_elems,
-                                          uint32_t tile_elems) {
-  using G = ZvcGeom<T>;
-  if (e0 + G::EPV <= bulk_elems) return *reinterpret_cast<const uint4*>(stage + e0 * G::W);
-  uint32_t w4[4] = {0, 0, 0, 0};
-  for (int i = 0; i < G::EPV; i++)
-    if (e0 + i < tile_elems) {
-      const uint32_t x = uint32_t(gsrc[e0 + i]);
-      if constexpr (sizeof(T) == 4) w4[i] = x;
-      else w4[i >> 1] |= x << ((i & 1) * 16);
-    }
-  return make_uint4(w4[0], w4[1], w4[2], w4[3]);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -110,6 +77,15 @@ constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 #define CSWAP_ZVC_MAX_BACKOFF 32
 #endif
 constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
+// 16-byte emit stores unrolled per lane
+#ifndef CSWAP_ZVC_EMIT_UNROLL
+#define CSWAP_ZVC_EMIT_UNROLL 2
+#endif
+constexpr int kEmitUnroll = CSWAP_ZVC_EMIT_UNROLL;
+// rows per batch of count_slab's loads
+#ifndef CSWAP_ZVC_BATCH
+#define CSWAP_ZVC_BATCH 16
+#endif
 // mbarrier waits sleep between tests (max ns): the producer refills a stage whose TMA load takes
 // ~1 us anyway; a resolver has LAG tile periods (~1.5 us each) before its offset is needed; the
 // polling consumer warp is on the critical path and sleeps least
@@ -118,6 +94,20 @@ constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
 #endif
 constexpr uint32_t kProducerSleep = 256 * CSWAP_ZVC_SLEEP, kResolverSleep = 128 * CSWAP_ZVC_SLEEP,
                    kConsumerSleep = 64 * CSWAP_ZVC_SLEEP;
+
+// the resolver handshakes (tile counted -> resolver; offset resolved -> consumers) on named
+// barriers (bar.arrive / bar.sync: a waiting warp issues nothing) instead of polled mbarriers
+// (ncu, f16 1 GiB: the polling loops were 39 % of all issued instructions)
+#ifndef CSWAP_ZVC_NAMED
+#define CSWAP_ZVC_NAMED 1
+#endif
+constexpr bool kNamedBars = CSWAP_ZVC_NAMED != 0;
+__device__ __forceinline__ void named_arrive(uint32_t id, uint32_t nthreads) {
+  asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+__device__ __forceinline__ void named_sync(uint32_t id, uint32_t nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
 
 #ifndef CSWAP_ZVC_DYNAMIC_TILES
 constexpr bool kStaticTiles = true;
@@ -139,16 +129,42 @@ struct CompressSmem {
   static constexpr uint32_t in_off = 0;
   static constexpr uint32_t bytes = S * TB + 128;  // dynamic: the stage ring (+ pad)
   static constexpr uint32_t static_bytes = S * G::WT * 4 + 1024;  // bitmap words, barriers, ...
-  static constexpr int ctas_per_sm = bytes + static_bytes <= 112 * 1024 ? 2 : 1;
+  // resident CTAs per SM allowed by shared memory (228 KiB per SM, 1 KiB reserved per CTA), max 4
+  static constexpr int by_smem = int((228u * 1024u) / (bytes + static_bytes + 1024u));
+  static constexpr int ctas_per_sm = by_smem > 4 ? 4 : (by_smem < 1 ? 1 : by_smem);
 };
 
-__device__ __forceinline__ uint32_t spread16(uint32_t x) {  // bit i -> bit 2i (i < 16)
-  x &= 0xFFFFu;
-  x = (x | (x << 8)) & 0x00FF00FFu;
-  x = (x | (x << 4)) & 0x0F0F0F0Fu;
-  x = (x | (x << 2)) & 0x33333333u;
-  x = (x | (x << 1)) & 0x55555555u;
-  return x;
+// Copy a slab's compacted non-zeros (cnt words of W bytes at shared sv) to dst: element stores up
+// to the destination's next 16-byte boundary, then 16-byte stores whose source is the smem slab
+// funnel-shifted by that head (k whole words + r bits, warp-uniform, so one of four unrolled
+// bodies runs), then the element tail.  Called by one whole warp.
+template <typename T>
+__device__ __forceinline__ void emit_words(const T* sv, uint32_t cnt, uint8_t* dst, int lane) {
+  T* d = reinterpret_cast<T*>(dst);
+  const uint32_t nbytes = cnt * sizeof(T);
+  const uint32_t h = umin32((16u - (uint32_t(reinterpret_cast<uintptr_t>(dst)) & 15u)) & 15u, nbytes);
+  const uint32_t nb = (nbytes - h) >> 4, tail = h + 16 * nb;
+  if (uint32_t(lane) < h / sizeof(T)) d[lane] = sv[lane];
+  if (uint32_t(lane) < (nbytes - tail) / sizeof(T)) d[tail / sizeof(T) + lane] = sv[tail / sizeof(T) + lane];
+  const uint32_t sa = uint32_t(__cvta_generic_to_shared(sv));
+  uint4* dv = reinterpret_cast<uint4*>(dst + h);
+  auto body = [&](auto kk) {
+    constexpr int k = decltype(kk)::value;
+    const uint32_t r = (h & 3u) * 8u;
+#pragma unroll kEmitUnroll
+    for (uint32_t q = lane; q < nb; q += 32) {
+      const uint4 A = lds_v4(sa + 16 * q), B = lds_v4(sa + 16 * q + 16);
+      const uint32_t w[8] = {A.x, A.y, A.z, A.w, B.x, B.y, B.z, B.w};
+      stg_stream(dv + q, make_uint4(__funnelshift_r(w[k], w[k + 1], r), __funnelshift_r(w[k + 1], w[k + 2], r),
+                                    __funnelshift_r(w[k + 2], w[k + 3], r), __funnelshift_r(w[k + 3], w[k + 4], r)));
+    }
+  };
+  switch (h >> 2) {
+    case 0: body(std::integral_constant<int, 0>{}); break;
+    case 1: body(std::integral_constant<int, 1>{}); break;
+    case 2: body(std::integral_constant<int, 2>{}); break;
+    default: body(std::integral_constant<int, 3>{}); break;
+  }
 }
 
 // S stages; CW consumer warps; the consumers count tile i and emit tile i - LAG (LAG = S - 2),
@@ -164,6 +180,9 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
   constexpr uint32_t SENT = 0xFFFFFFFFu;
   constexpr int kProducerWarp = CW;
   constexpr int LAG = S - 2;
+  // named barriers: 0 = __syncthreads, 1 = consumer_sync, then per stage count / offset
+  constexpr uint32_t kBarCnt0 = 2, kBarOff0 = 2 + S;
+  static_assert(kBarOff0 + S <= 16, "named barrier ids");
   constexpr int PW = G::TILE / CW;   // elements per consumer warp (slab) per tile
   constexpr int WPW = G::WT / CW;    // bitmap words per slab
   static_assert(LAG >= 1 && PW % 256 == 0, "compress geometry");
@@ -238,7 +257,8 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     for (uint32_t i = r;; i += S) {
       const int s = r;
       long long c0 = clock64();
-      mbar_wait_sleep(&bar_cnt[s], (i / S) & 1, kResolverSleep);
+      if (kNamedBars) named_sync(kBarCnt0 + s, 64);
+      else mbar_wait_sleep(&bar_cnt[s], (i / S) & 1, kResolverSleep);
       long long c1 = clock64();
       if (lane == 0) ZPROF_ADD(2, c1 - c0);
       const uint32_t nnz = s_nnz[s];
@@ -318,9 +338,10 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         ZPROF_ADD(3, clock64() - c1);
         s_off[s] = excl;
         s_fs[s] = fstart;
-        mbar_arrive(&bar_off[s]);
+        if (!kNamedBars) mbar_arrive(&bar_off[s]);
       }
       __syncwarp();
+      if (kNamedBars) named_arrive(kBarOff0 + s, 32 * (CW + 1));
     }
     return;
   }
@@ -354,7 +375,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     // non-zeros are compacted in place to the start of the slab (a row's writes land at or
     // before the row, and every row of a batch is loaded before any of its writes).
     // Rows go in batches of 16 so the batch's loads issue back to back.
-    constexpr int B = EROWS < 16 ? EROWS : 16;
+    constexpr int B = EROWS < CSWAP_ZVC_BATCH ? EROWS : CSWAP_ZVC_BATCH;
     const uint32_t e0 = warp * PW + lane;
     T* sv = reinterpret_cast<T*>(stage) + warp * PW;
     uint32_t tot = 0;
@@ -375,36 +396,9 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     return tot;
   };
 
-  // copy the slab's compacted non-zeros (count_slab) to the container: element stores up to the
-  // destination's next 16-byte boundary, then 16-byte stores whose source is the smem slab
-  // funnel-shifted by that head (k whole words + r bits, warp-uniform), then the element tail
+  // copy the slab's compacted non-zeros (count_slab) to the container (emit_words)
   auto emit_slab = [&](const uint8_t* stage, uint32_t cnt, uint8_t* dst) {
-    const T* sv = reinterpret_cast<const T*>(stage) + warp * PW;
-    T* d = reinterpret_cast<T*>(dst);
-    const uint32_t nbytes = cnt * G::W;
-    const uint32_t h = umin32((16u - (uint32_t(reinterpret_cast<uintptr_t>(dst)) & 15u)) & 15u, nbytes);
-    const uint32_t nb = (nbytes - h) >> 4, tail = h + 16 * nb;
-    if (uint32_t(lane) < h / G::W) d[lane] = sv[lane];
-    if (uint32_t(lane) < (nbytes - tail) / G::W) d[tail / G::W + lane] = sv[tail / G::W + lane];
-    const uint32_t sa = uint32_t(__cvta_generic_to_shared(sv));
-    uint4* dv = reinterpret_cast<uint4*>(dst + h);
-    auto body = [&](auto kk) {
-      constexpr int k = decltype(kk)::value;
-      const uint32_t r = (h & 3u) * 8u;
-#pragma unroll 2
-      for (uint32_t q = lane; q < nb; q += 32) {
-        const uint4 A = lds_v4(sa + 16 * q), B = lds_v4(sa + 16 * q + 16);
-        const uint32_t w[8] = {A.x, A.y, A.z, A.w, B.x, B.y, B.z, B.w};
-        stg_stream(dv + q, make_uint4(__funnelshift_r(w[k], w[k + 1], r), __funnelshift_r(w[k + 1], w[k + 2], r),
-                                      __funnelshift_r(w[k + 2], w[k + 3], r), __funnelshift_r(w[k + 3], w[k + 4], r)));
-      }
-    };
-    switch (h >> 2) {
-      case 0: body(std::integral_constant<int, 0>{}); break;
-      case 1: body(std::integral_constant<int, 1>{}); break;
-      case 2: body(std::integral_constant<int, 2>{}); break;
-      default: body(std::integral_constant<int, 3>{}); break;
-    }
+    emit_words<T>(reinterpret_cast<const T*>(stage) + warp * PW, cnt, dst, lane);
   };
 
   auto count = [&](uint32_t i, uint32_t t) {
@@ -427,14 +421,19 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       atomicAdd(reinterpret_cast<unsigned long long*>(sc.aux2 + k), (1ull << 40) + tot);
       atomicAdd(reinterpret_cast<unsigned long long*>(sc.aux2 + K + uint64_t(k) * gpf + j / 32), (1ull << 40) + tot);
       s_nnz[s] = tot;
-      mbar_arrive(&bar_cnt[s]);
+      if (!kNamedBars) mbar_arrive(&bar_cnt[s]);
+    }
+    if (kNamedBars && warp == 0) {
+      __syncwarp();
+      named_arrive(kBarCnt0 + s, 64);
     }
   };
 
   auto emit = [&](uint32_t i, uint32_t t) {
     const int s = i % S;
     long long c0 = clock64();
-    group_wait(&bar_off[s], (i / S) & 1);
+    if (kNamedBars) named_sync(kBarOff0 + s, 32 * (CW + 1));
+    else group_wait(&bar_off[s], (i / S) & 1);
     if (tid == 0) ZPROF_ADD(5, clock64() - c0);
     long long c2 = clock64();
     const uint64_t g0 = s_off[s], fstart = s_fs[s];
@@ -492,8 +491,12 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       if (tid == 0) {
         for (uint32_t i2 = i; i2 < i + S; i2++) {
           s_nnz[i2 % S] = SENT;
-          mbar_arrive(&bar_cnt[i2 % S]);
+          if (!kNamedBars) mbar_arrive(&bar_cnt[i2 % S]);
         }
+      }
+      if (kNamedBars && warp == 0) {
+        __syncwarp();
+        for (int s2 = 0; s2 < S; s2++) named_arrive(kBarCnt0 + s2, 64);
       }
       break;
     }
@@ -834,6 +837,7 @@ static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uin
 }
 
 // compress configuration (stages x tile bytes): cswap_set_zvc_launch, else CSWAP_ZVC_CFG, else 0
+constexpr int kMaxVariant = 8;
 static int compress_cfg() {
   const int v = g_zvc_variant.load(std::memory_order_relaxed);
   if (v >= 0) return v;
@@ -841,13 +845,13 @@ static int compress_cfg() {
   if (c < 0) {
     const char* e = getenv("CSWAP_ZVC_CFG");
     c = e ? atoi(e) : 0;
-    if (c < 0 || c > 3) c = 0;
+    if (c < 0 || c > kMaxVariant) c = 0;
   }
   return c;
 }
 
 bool zvc_set_launch(uint32_t grid, int variant) {
-  if (variant < -1 || variant > 3) return false;
+  if (variant < -1 || variant > kMaxVariant) return false;
   g_zvc_grid.store(grid);
   g_zvc_variant.store(variant);
   return true;
@@ -860,6 +864,15 @@ static cudaError_t launch_compress_t(const void* in, uint64_t n, uint64_t F, uin
     case 1: return launch_compress_s<T, 6, 8, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
     case 2: return launch_compress_s<T, 5, 8, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
     case 3: return launch_compress_s<T, 4, 8, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    // one CTA per SM with 16 consumer warps and a deeper ring (LAG = S - 2 tile periods of slack
+    // for the offsets, which wait for every earlier tile's count)
+    case 4: return launch_compress_s<T, 6, 16, 32768>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    case 5: return launch_compress_s<T, 5, 16, 32768>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    case 6: return launch_compress_s<T, 4, 16, 32768>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    // more, smaller CTAs per SM: 4 consumer warps per 16 KiB tile, so per-tile latencies
+    // (barriers, the offset wait) of 3-4 resident tiles overlap
+    case 7: return launch_compress_s<T, 3, 4, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    case 8: return launch_compress_s<T, 4, 4, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
     default: return launch_compress_s<T, 3, 8, 32768>(in, n, F, out, out_size, sc, epoch, dtype, st);
   }
 }

@@ -11,7 +11,11 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libcswap.so")
+# CSWAP_LIB_VARIANT=<tag> loads variants/libcswap_<tag>.so, an A/B build of the same sources with
+# different compile-time switches (tools/build_variants.py); default: the in-tree libcswap.so
+_VARIANT = os.environ.get("CSWAP_LIB_VARIANT") or None
+LIB_PATH = (os.path.join(_HERE, "variants", f"libcswap_{_VARIANT}.so") if _VARIANT
+            else os.path.join(_HERE, "libcswap.so"))
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_cluster_chenhzchysc21_b200.build`"
                       " (there is no CPU fallback)")

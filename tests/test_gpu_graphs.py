@@ -91,7 +91,8 @@ def test_plain_launch_path_matches():
     assert r.returncode == 0 and "plain ok" in r.stdout, r.stderr[-3000:]
 
 
-@pytest.mark.parametrize("grid,variant", [(1, 0), (7, 1), (148, 2), (296, 3), (0, -1)])
+@pytest.mark.parametrize("grid,variant", [(1, 0), (7, 1), (148, 2), (296, 3), (0, 4), (5, 5),
+                                           (148, 6), (0, 7), (300, 8), (0, -1)])
 def test_zvc_launch_config_keeps_bytes(C, grid, variant):
     """cswap_set_zvc_launch changes only how the persistent compress runs, never its bytes."""
     n = (1 << 21) + 333
@@ -106,7 +107,7 @@ def test_zvc_launch_config_keeps_bytes(C, grid, variant):
 
 def test_zvc_launch_config_rejects_bad_variant(C):
     with pytest.raises(C.CswapError):
-        C.set_zvc_launch(0, 4)
+        C.set_zvc_launch(0, 9)
 
 
 def test_timing_records_carry_device_clock(C):
