@@ -4,6 +4,7 @@
 // the single-pass codec kernels, and small PTX wrappers (acquire/release at .gpu scope).
 #pragma once
 #include <cstdint>
+#include <type_traits>
 #include <cuda_runtime.h>
 
 namespace cswap {
@@ -288,6 +289,41 @@ __device__ __forceinline__ void stg_stream(uint4* p, uint4 v) {
   asm volatile("st.global.L1::no_allocate.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
                "r"(v.w)
                : "memory");
+}
+
+// Copy a slab's compacted non-zeros (cnt words of W bytes at shared sv) to dst: element stores up
+// to the destination's next 16-byte boundary, then 16-byte stores whose source is the smem slab
+// funnel-shifted by that head (k whole words + r bits, warp-uniform, so one of four unrolled
+// bodies runs), then the element tail.  Called by `stride` threads (a warp: stride 32, idx =
+// lane; a block: stride blockDim.x, idx = threadIdx.x); sv is 16-byte aligned with >= 16
+// readable bytes past the last word.
+template <typename T>
+__device__ __forceinline__ void emit_words(const T* sv, uint32_t cnt, uint8_t* dst, uint32_t idx, uint32_t stride) {
+  T* d = reinterpret_cast<T*>(dst);
+  const uint32_t nbytes = cnt * sizeof(T);
+  const uint32_t h = umin32((16u - (uint32_t(reinterpret_cast<uintptr_t>(dst)) & 15u)) & 15u, nbytes);
+  const uint32_t nb = (nbytes - h) >> 4, tail = h + 16 * nb;
+  if (idx < h / sizeof(T)) d[idx] = sv[idx];
+  if (idx < (nbytes - tail) / sizeof(T)) d[tail / sizeof(T) + idx] = sv[tail / sizeof(T) + idx];
+  const uint32_t sa = uint32_t(__cvta_generic_to_shared(sv));
+  uint4* dv = reinterpret_cast<uint4*>(dst + h);
+  auto body = [&](auto kk) {
+    constexpr int k = decltype(kk)::value;
+    const uint32_t r = (h & 3u) * 8u;
+#pragma unroll 2
+    for (uint32_t q = idx; q < nb; q += stride) {
+      const uint4 A = lds_v4(sa + 16 * q), B = lds_v4(sa + 16 * q + 16);
+      const uint32_t w[8] = {A.x, A.y, A.z, A.w, B.x, B.y, B.z, B.w};
+      stg_stream(dv + q, make_uint4(__funnelshift_r(w[k], w[k + 1], r), __funnelshift_r(w[k + 1], w[k + 2], r),
+                                    __funnelshift_r(w[k + 2], w[k + 3], r), __funnelshift_r(w[k + 3], w[k + 4], r)));
+    }
+  };
+  switch (h >> 2) {
+    case 0: body(std::integral_constant<int, 0>{}); break;
+    case 1: body(std::integral_constant<int, 1>{}); break;
+    case 2: body(std::integral_constant<int, 2>{}); break;
+    default: body(std::integral_constant<int, 3>{}); break;
+  }
 }
 
 // Write the 64-byte container header (one thread).

@@ -77,11 +77,6 @@ constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 #define CSWAP_ZVC_MAX_BACKOFF 32
 #endif
 constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
-// 16-byte emit stores unrolled per lane
-#ifndef CSWAP_ZVC_EMIT_UNROLL
-#define CSWAP_ZVC_EMIT_UNROLL 2
-#endif
-constexpr int kEmitUnroll = CSWAP_ZVC_EMIT_UNROLL;
 // rows per batch of count_slab's loads
 #ifndef CSWAP_ZVC_BATCH
 #define CSWAP_ZVC_BATCH 16
@@ -133,39 +128,6 @@ struct CompressSmem {
   static constexpr int by_smem = int((228u * 1024u) / (bytes + static_bytes + 1024u));
   static constexpr int ctas_per_sm = by_smem > 4 ? 4 : (by_smem < 1 ? 1 : by_smem);
 };
-
-// Copy a slab's compacted non-zeros (cnt words of W bytes at shared sv) to dst: element stores up
-// to the destination's next 16-byte boundary, then 16-byte stores whose source is the smem slab
-// funnel-shifted by that head (k whole words + r bits, warp-uniform, so one of four unrolled
-// bodies runs), then the element tail.  Called by one whole warp.
-template <typename T>
-__device__ __forceinline__ void emit_words(const T* sv, uint32_t cnt, uint8_t* dst, int lane) {
-  T* d = reinterpret_cast<T*>(dst);
-  const uint32_t nbytes = cnt * sizeof(T);
-  const uint32_t h = umin32((16u - (uint32_t(reinterpret_cast<uintptr_t>(dst)) & 15u)) & 15u, nbytes);
-  const uint32_t nb = (nbytes - h) >> 4, tail = h + 16 * nb;
-  if (uint32_t(lane) < h / sizeof(T)) d[lane] = sv[lane];
-  if (uint32_t(lane) < (nbytes - tail) / sizeof(T)) d[tail / sizeof(T) + lane] = sv[tail / sizeof(T) + lane];
-  const uint32_t sa = uint32_t(__cvta_generic_to_shared(sv));
-  uint4* dv = reinterpret_cast<uint4*>(dst + h);
-  auto body = [&](auto kk) {
-    constexpr int k = decltype(kk)::value;
-    const uint32_t r = (h & 3u) * 8u;
-#pragma unroll kEmitUnroll
-    for (uint32_t q = lane; q < nb; q += 32) {
-      const uint4 A = lds_v4(sa + 16 * q), B = lds_v4(sa + 16 * q + 16);
-      const uint32_t w[8] = {A.x, A.y, A.z, A.w, B.x, B.y, B.z, B.w};
-      stg_stream(dv + q, make_uint4(__funnelshift_r(w[k], w[k + 1], r), __funnelshift_r(w[k + 1], w[k + 2], r),
-                                    __funnelshift_r(w[k + 2], w[k + 3], r), __funnelshift_r(w[k + 3], w[k + 4], r)));
-    }
-  };
-  switch (h >> 2) {
-    case 0: body(std::integral_constant<int, 0>{}); break;
-    case 1: body(std::integral_constant<int, 1>{}); break;
-    case 2: body(std::integral_constant<int, 2>{}); break;
-    default: body(std::integral_constant<int, 3>{}); break;
-  }
-}
 
 // S stages; CW consumer warps; the consumers count tile i and emit tile i - LAG (LAG = S - 2),
 // so a tile's offset has LAG count phases of slack to resolve.
@@ -398,7 +360,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
 
   // copy the slab's compacted non-zeros (count_slab) to the container (emit_words)
   auto emit_slab = [&](const uint8_t* stage, uint32_t cnt, uint8_t* dst) {
-    emit_words<T>(reinterpret_cast<const T*>(stage) + warp * PW, cnt, dst, lane);
+    emit_words<T>(reinterpret_cast<const T*>(stage) + warp * PW, cnt, dst, lane, 32);
   };
 
   auto count = [&](uint32_t i, uint32_t t) {
