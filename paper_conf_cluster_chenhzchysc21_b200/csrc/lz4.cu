@@ -73,6 +73,7 @@ __device__ __forceinline__ uint32_t emit_seq(uint8_t* out, uint32_t op, const ui
 // shared memory, so 4 blocks per CTA and ~28 parsing warps per SM hide each other's latency
 // (staging the 64 KiB block limited an SM to 3 warps: 7.6 GB/s at s = 0.5).
 constexpr int kLz4Warps = 4;
+constexpr uint32_t kLz4Ring = 4096;  // decode: recent-output ring per warp (power of two, >= 32)
 
 __device__ __forceinline__ uint32_t le32_g(const uint8_t* s, uint32_t p) {  // s 16-aligned; p+8 <= block end
   const uint32_t* w = reinterpret_cast<const uint32_t*>(s);
@@ -259,10 +260,16 @@ __global__ void __launch_bounds__(32 * kLz4Warps) lz4_decode_kernel(const uint8_
                                                                     uint64_t n, int w, uint64_t F, uint32_t B,
                                                                     uint32_t bpf, uint32_t k0, uint32_t nslots,
                                                                     Scratch sc, uint32_t* err) {
+  // the warp's last kLz4Ring output bytes (ring indexed by output position): match sources within
+  // that distance are read from shared memory, not back from L2 (an L2 round trip per match
+  // bounded the decode at ~55 GB/s for ReLU data, whose matches are mostly a few bytes back)
+  __shared__ __align__(16) uint8_t s_rings[kLz4Warps][kLz4Ring];
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const int lane = threadIdx.x & 31;
   const uint32_t slot = blockIdx.x * kLz4Warps + (threadIdx.x >> 5);
   if (slot >= nslots) return;
+  uint8_t* ring = s_rings[threadIdx.x >> 5];
+  constexpr uint32_t RM = kLz4Ring - 1;
   const uint32_t k = k0 + slot / bpf, b = slot % bpf;
   const uint64_t fbytes = frame_len(n, F, k) * uint64_t(w);
   const uint32_t nb = uint32_t(cdiv(fbytes, B));
@@ -292,7 +299,11 @@ __global__ void __launch_bounds__(32 * kLz4Warps) lz4_decode_kernel(const uint8_
       if (bad) break;
     }
     if (ip + nlit > cs || op + nlit > L) { bad = true; break; }
-    for (uint32_t q = lane; q < nlit; q += 32) dst[op + q] = __ldg(ip0 + ip + q);
+    for (uint32_t q = lane; q < nlit; q += 32) {
+      const uint8_t x = __ldg(ip0 + ip + q);
+      dst[op + q] = x;
+      ring[(op + q) & RM] = x;
+    }
     ip += nlit;
     op += nlit;
     if (ip == cs) break;  // last sequence: literals only
@@ -313,17 +324,26 @@ __global__ void __launch_bounds__(32 * kLz4Warps) lz4_decode_kernel(const uint8_
     if (offset == 0 || offset > op || op + mlen > L) { bad = true; break; }
     __syncwarp();  // the match source may have been written by other lanes
     if (offset >= 32) {  // non-overlapping within a 32-byte step
+      const bool near = offset <= kLz4Ring;  // source still in the ring
       for (uint32_t q = 0; q < mlen; q += 32) {
-        if (q + lane < mlen) dst[op + q + lane] = ld_cg_u8(dst + op + q + lane - offset);
+        if (q + lane < mlen) {
+          const uint32_t o = op + q + lane;
+          const uint8_t x = near ? ring[(o - offset) & RM] : ld_cg_u8(dst + o - offset);
+          dst[o] = x;
+          ring[o & RM] = x;
+        }
         __syncwarp();
       }
     } else {  // short offset: the match repeats the last `offset` bytes
       const uint32_t base = op - offset;
-      const uint32_t pat = lane < int(offset) ? ld_cg_u8(dst + base + lane) : 0u;
+      const uint32_t pat = lane < int(offset) ? ring[(base + lane) & RM] : 0u;
       for (uint32_t q0 = 0; q0 < mlen; q0 += 32) {  // whole-warp iterations: every lane shuffles
         const uint32_t q = q0 + lane;
         const uint32_t v = __shfl_sync(0xffffffffu, pat, q % offset);
-        if (q < mlen) dst[op + q] = uint8_t(v);
+        if (q < mlen) {
+          dst[op + q] = uint8_t(v);
+          ring[(op + q) & RM] = uint8_t(v);
+        }
       }
     }
     op += mlen;
