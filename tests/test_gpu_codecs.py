@@ -105,3 +105,37 @@ def test_probe_matches_oracle(C):
             d = G.to_dev(x)
             got = C.probe(d, n, dtype).tuple()
             assert got == O.probe(x, dtype)
+
+
+def _lz4_offset_case(gap: int, repeat: bool) -> np.ndarray:
+    """3 LZ4 blocks of incompressible words; in each, a periodic run of period `gap` (gap < 96),
+    or a random 96-byte pattern, zeros, and the pattern again `gap` bytes after the first copy
+    (positions inside the zero run's match are not inserted, so the first copy stays
+    in the hash table).  repeat=False replaces the second copy by other random bytes (control)."""
+    rng = np.random.default_rng(gap)
+    x = rng.integers(1, 2**32, size=3 * 16384, dtype=np.uint64).astype(np.uint32)
+    raw = x.view(np.uint8)
+    pat, other = rng.integers(0, 256, size=(2, 96), dtype=np.uint8)
+    for blk in range(3):
+        p0 = blk * 65536 + 1000
+        if gap < 96:
+            raw[p0:p0 + 256] = np.resize(pat[:gap], 256) if repeat else np.resize(other, 256)
+        else:
+            raw[p0:p0 + 96] = pat
+            raw[p0 + 96:p0 + gap] = 0
+            raw[p0 + gap:p0 + gap + 96] = pat if repeat else other
+    return x
+
+
+@pytest.mark.parametrize("gap", [3, 31, 32, 33, 4000, 4096, 4097, 10000, 60000])
+def test_lz4_match_offsets(C, gap):
+    """Every match-offset class of the LZ4 decoder: overlapping short offsets (< 32 bytes,
+    pattern replication), offsets served by the warp's 4 KiB recent-output ring, and offsets
+    beyond it (read back from global memory).  The GPU must produce the oracle's bytes and
+    decode them; the oracle's container is smaller than the control's, i.e. the repeats at
+    distance `gap` were parsed as matches."""
+    x = _lz4_offset_case(gap, True)
+    ref = O.compress(x, O.LZ4, O.F32, F=1 << 22, param=65536)
+    ctl = O.compress(_lz4_offset_case(gap, False), O.LZ4, O.F32, F=1 << 22, param=65536)
+    assert len(ref) + 3 * 50 < len(ctl)
+    check_parity(C, x, O.LZ4, O.F32)
