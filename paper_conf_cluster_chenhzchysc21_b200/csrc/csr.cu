@@ -186,6 +186,9 @@ cudaError_t launch_csr_compress(const void* in, uint64_t n, int w, uint64_t F, u
 // ------------------------------------------------------------------------------------------
 // decompress
 // ------------------------------------------------------------------------------------------
+#ifndef CSWAP_CSR_UNROLL
+#define CSWAP_CSR_UNROLL 4
+#endif
 template <typename T>
 __global__ void __launch_bounds__(kThreads) csr_expand_kernel(const uint8_t* __restrict__ in, T* __restrict__ outp,
                                                               uint64_t n, uint64_t F, uint32_t tpf, uint32_t C,
@@ -243,13 +246,36 @@ __global__ void __launch_bounds__(kThreads) csr_expand_kernel(const uint8_t* __r
         }
         q1 = lo;
       }
-      for (uint64_t q = q0 + lane; q < q1; q += 32) {
-        const uint32_t c = col[q];
-        if (c >= width || (q > a && col[q - 1] >= c)) {
-          bad = true;
-          continue;
+      // U x 32 (col, value) pairs per step, all loads issued before the first use (the loop
+      // was one dependent DRAM round trip per 32 pairs); the ascending-column check takes the
+      // predecessor from the neighbouring lane, and from memory only for the window's first pair
+      constexpr int U = CSWAP_CSR_UNROLL;
+      uint32_t prev = (q0 > a && q0 < q1) ? col[q0 - 1] : 0u;  // column before the window
+      bool has_prev = q0 > a;
+      for (uint64_t qb = q0; qb < q1; qb += 32 * U) {
+        uint32_t cv[U];
+        T vv[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          const uint64_t q = qb + uint64_t(u) * 32 + lane;
+          cv[u] = q < q1 ? col[q] : 0u;
+          vv[u] = q < q1 ? val[q] : T(0);
         }
-        if (c >= c_lo && c < c_hi) s_x[rs + c - p.tin] = val[q];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          const uint64_t q = qb + uint64_t(u) * 32 + lane;
+          const uint32_t up = __shfl_up_sync(0xffffffffu, cv[u], 1);
+          const uint32_t last = __shfl_sync(0xffffffffu, cv[u], 31);
+          const uint32_t pc = lane ? up : prev;
+          const bool hp = lane ? true : has_prev;
+          if (q < q1) {
+            const uint32_t c = cv[u];
+            if (c >= width || (hp && pc >= c)) bad = true;
+            else if (c >= c_lo && c < c_hi) s_x[rs + c - p.tin] = vv[u];
+          }
+          prev = last;
+          has_prev = true;
+        }
       }
     }
     if (bad) s_bad = 1;
