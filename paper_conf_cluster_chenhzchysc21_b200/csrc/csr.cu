@@ -14,6 +14,11 @@
 
 namespace cswap {
 
+// rows of 32 elements per batch of the emit pass's global loads
+#ifndef CSWAP_CSR_EMIT_BATCH
+#define CSWAP_CSR_EMIT_BATCH 8
+#endif
+
 template <typename T>
 __global__ void __launch_bounds__(kThreads) csr_count_kernel(const T* __restrict__ in, uint64_t n, uint64_t F,
                                                              uint32_t tpf, Scratch sc) {
@@ -85,7 +90,7 @@ __global__ void __launch_bounds__(kThreads) csr_emit_kernel(const T* __restrict_
   const uint32_t lt = (1u << lane) - 1u;
   // pass 1: per-warp counts (warp w owns elements [w*PER_WARP, (w+1)*PER_WARP) as rows of 32)
   // rows are loaded 8 at a time before their ballots (independent loads in flight)
-  constexpr int B = 8;
+  constexpr int B = G::ROWS < CSWAP_CSR_EMIT_BATCH ? G::ROWS : CSWAP_CSR_EMIT_BATCH;
   const bool full = p.te == G::TILE;
   uint32_t cnt = 0;
 #pragma unroll 1
