@@ -402,7 +402,7 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
   CU(cudaMalloc(&b.sc.aux2, aux * 8));
   CU(cudaMalloc(&b.sc.err, 64));
   CU(cudaMalloc(&b.sc.tbuf, tiles * 8));
-  CU(cudaMalloc(&b.sc.tbuf2, tiles * 8));
+  CU(cudaMalloc(&b.sc.tbuf2, tiles * 32));  // 32 B per tile: CSR keeps 8 u32 slab counts
   CU(cudaMalloc(&b.sc.aux3, aux * 8));
   CU(cudaMemset(b.sc.status, 0, tiles * 8));
   CU(cudaMemset(b.sc.tickets, 0, kEpochs * 4));

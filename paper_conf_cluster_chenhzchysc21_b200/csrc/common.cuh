@@ -36,7 +36,7 @@ struct Scratch {
   uint64_t* aux2;         // second per-frame / per-tile array
   uint32_t* err;          // device error word (first error wins)
   uint64_t* tbuf;         // per-tile u64 array for multi-kernel codecs (never epoch-tagged)
-  uint64_t* tbuf2;        // second per-tile u64 array
+  uint64_t* tbuf2;        // second per-tile array, 32 bytes per tile (u64, or CSR: u32[8] slab counts)
   uint64_t* aux3;         // third per-frame u64 array (run / non-zero totals)
   uint64_t cap_tiles, cap_aux;
 };

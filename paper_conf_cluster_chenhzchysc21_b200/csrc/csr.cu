@@ -27,13 +27,16 @@ __global__ void __launch_bounds__(kThreads) csr_count_kernel(const T* __restrict
   const uint32_t t = blockIdx.x;
   const TilePos p = tile_pos<T>(t, n, F, tpf);
   const T* src = in + uint64_t(p.k) * F + p.tin;
+  // per-warp counts of the emit kernel's slabs (warp w: elements [w*PER_WARP, (w+1)*PER_WARP)),
+  // kept in tbuf2 so that the emit pass reads the tile once
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   uint32_t c = 0;
   if (p.te == G::TILE) {  // full tile: 16-byte loads, all in flight
     constexpr int V = G::TILE * int(sizeof(T)) / 16 / kThreads;
-    const uint4* s4 = reinterpret_cast<const uint4*>(src);
+    const uint4* s4 = reinterpret_cast<const uint4*>(src) + warp * (32 * V);
     uint4 q[V];
 #pragma unroll
-    for (int i = 0; i < V; i++) q[i] = __ldg(s4 + threadIdx.x + i * kThreads);
+    for (int i = 0; i < V; i++) q[i] = __ldg(s4 + lane + i * 32);
 #pragma unroll
     for (int i = 0; i < V; i++) {
       if constexpr (sizeof(T) == 4) {
@@ -45,8 +48,11 @@ __global__ void __launch_bounds__(kThreads) csr_count_kernel(const T* __restrict
       }
     }
   } else {
-    for (uint32_t e = threadIdx.x; e < p.te; e += blockDim.x) c += src[e] != 0;
+    const uint32_t e1 = umin32(p.te, (warp + 1) * G::PER_WARP);
+    for (uint32_t e = warp * G::PER_WARP + lane; e < e1; e += 32) c += src[e] != 0;
   }
+  const uint32_t wc = __reduce_add_sync(0xffffffffu, c);
+  if (lane == 0) reinterpret_cast<uint32_t*>(sc.tbuf2)[uint64_t(t) * kWarps + warp] = wc;
   c = block_sum_u32(c, s_tmp);
   if (threadIdx.x == 0) sc.tbuf[t] = c;
 }
@@ -88,23 +94,10 @@ __global__ void __launch_bounds__(kThreads) csr_emit_kernel(const T* __restrict_
   const TilePos p = tile_pos<T>(t, n, F, tpf);
   const T* src = in + uint64_t(p.k) * F + p.tin;
   const uint32_t lt = (1u << lane) - 1u;
-  // pass 1: per-warp counts (warp w owns elements [w*PER_WARP, (w+1)*PER_WARP) as rows of 32)
-  // rows are loaded 8 at a time before their ballots (independent loads in flight)
+  // slab offsets inside the tile from the count kernel's per-warp counts (tbuf2)
   constexpr int B = G::ROWS < CSWAP_CSR_EMIT_BATCH ? G::ROWS : CSWAP_CSR_EMIT_BATCH;
   const bool full = p.te == G::TILE;
-  uint32_t cnt = 0;
-#pragma unroll 1
-  for (int m0 = 0; m0 < G::ROWS; m0 += B) {
-    T v[B];
-#pragma unroll
-    for (int u = 0; u < B; u++) {
-      const uint32_t e = warp * G::PER_WARP + 32 * (m0 + u) + lane;
-      v[u] = (full || e < p.te) ? src[e] : T(0);
-    }
-#pragma unroll
-    for (int u = 0; u < B; u++) cnt += __popc(__ballot_sync(0xffffffffu, v[u] != 0));
-  }
-  if (lane == 0) s_wcnt[warp] = cnt;
+  if (tid < kWarps) s_wcnt[tid] = reinterpret_cast<const uint32_t*>(sc.tbuf2)[uint64_t(t) * kWarps + tid];
   __syncthreads();
   if (tid == 0) {
     uint32_t a = 0;
