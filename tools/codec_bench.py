@@ -16,7 +16,7 @@ sys.path.insert(0, ROOT)
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--codecs", default="zvc")
-    ap.add_argument("--mib", type=int, default=1024)
+    ap.add_argument("--mib", type=float, default=1024, help="tensor size in MiB (fractions allowed: 0.0625 = 64 KiB)")
     ap.add_argument("--s", default="0.5")
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--dtype", default="f32")
@@ -32,7 +32,7 @@ def main():
     names = {"none": C.NONE, "zvc": C.ZVC, "rle": C.RLE, "csr": C.CSR, "lz4": C.LZ4}
     dtype = {"f32": C.F32, "f16": C.F16, "bf16": C.BF16}[a.dtype]
     w = C.WIDTH[dtype]
-    n = a.mib * 2**20 // w
+    n = int(a.mib * 2**20) // w
     peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
@@ -60,7 +60,7 @@ def main():
             def decomp(nb):
                 C.decompress(buf, nb, y, n, dtype, codec, err=err)
 
-            res = {"codec": cname, "s": s, "MiB": a.mib, "dtype": a.dtype}
+            res = {"codec": cname, "s": s, "MiB": a.mib, "dtype": a.dtype, "kind": a.kind}
             for label, fn in (("compress", comp), ("decompress", None)):
                 if fn is None:
                     nb = int(size.item())
