@@ -277,14 +277,16 @@ __global__ void __launch_bounds__(32 * kLz4Warps) lz4_decode_kernel(const uint8_
   const uint32_t L = uint32_t(umin64(B, fbytes - uint64_t(b) * B));
   const uint64_t blk = uint64_t(k) * bpf + b;
   const uint64_t fstart = sc.aux[k], fb = sc.aux2[k];
-  const uint64_t cs = sc.tbuf[blk];
+  const uint64_t cs64 = sc.tbuf[blk];
   const uint64_t start = a16(4ull * nb) + sc.tbuf2[blk];
-  bool bad = start + cs > fb;
+  // a valid block is at most LZ4's bound for L bytes, so the parse runs on 32-bit offsets
+  bool bad = start + cs64 > fb || cs64 > uint64_t(L) + L / 255 + 16;
+  const uint32_t cs = bad ? 0u : uint32_t(cs64);
   const uint8_t* ip0 = in + fstart + start;
   uint8_t* dst = outp + uint64_t(k) * F * w + uint64_t(b) * B;
-  uint64_t ip = 0;
+  uint32_t ip = 0;
   uint32_t op = 0;
-  auto rd = [&](uint64_t at) -> uint32_t { return at < cs ? __ldg(ip0 + at) : 0u; };
+  auto rd = [&](uint32_t at) -> uint32_t { return at < cs ? __ldg(ip0 + at) : 0u; };
   while (!bad) {
     if (ip >= cs) { bad = true; break; }
     const uint32_t token = rd(ip++);
