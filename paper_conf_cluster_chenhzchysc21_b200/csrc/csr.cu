@@ -122,30 +122,61 @@ __global__ void __launch_bounds__(kThreads) csr_emit_kernel(const T* __restrict_
   const uint64_t row0 = p.tin / C;
   const bool pow2 = (C & (C - 1)) == 0;
   const int csh = __ffs(int(C)) - 1;
+  // tile-local ranks (u32) against section pointers advanced to the tile's first non-zero
+  uint32_t* tcol = col_idx + tile_off;
+  T* tval = values + tile_off;
+  uint32_t lpre = uint32_t(pre - tile_off);
+  if (full && pow2 && C >= 32) {
+    // fast path: a row of 32 elements never straddles a CSR row (C = 2^k >= 32 and the tile
+    // starts on a multiple of 32), so its columns are colbase + lane and only lane 31 can end
+    // a CSR row: per element a ballot rank, the column add and the two stores
 #pragma unroll 1
-  for (int m0 = 0; m0 < G::ROWS; m0 += B) {
-    T vb[B];
+    for (int m0 = 0; m0 < G::ROWS; m0 += B) {
+      T vb[B];
 #pragma unroll
-    for (int u = 0; u < B; u++) {
-      const uint32_t e = warp * G::PER_WARP + 32 * (m0 + u) + lane;
-      vb[u] = (full || e < p.te) ? src[e] : T(0);
-    }
+      for (int u = 0; u < B; u++) vb[u] = src[warp * G::PER_WARP + 32 * (m0 + u) + lane];
 #pragma unroll
-    for (int u = 0; u < B; u++) {
-      const uint32_t e = warp * G::PER_WARP + 32 * (m0 + u) + lane;
-      const T v = vb[u];
-      const uint32_t b = __ballot_sync(0xffffffffu, v != 0);
-      const uint64_t rank = pre + __popc(b & lt);
-      const uint32_t x = cbase + e;
-      const uint32_t ro = pow2 ? x >> csh : x / C;
-      const uint32_t col = x - ro * C;
-      if (v != 0) {
-        col_idx[rank] = col;
-        values[rank] = v;
+      for (int u = 0; u < B; u++) {
+        const uint32_t e0 = warp * G::PER_WARP + 32 * (m0 + u);
+        const uint32_t x0 = cbase + e0;
+        const T v = vb[u];
+        const uint32_t b = __ballot_sync(0xffffffffu, v != 0);
+        const uint32_t r = lpre + __popc(b & lt);
+        if (v != 0) {
+          tcol[r] = (x0 & (C - 1)) + lane;
+          tval[r] = v;
+        }
+        lpre += __popc(b);
+        if (lane == 31 && (((x0 + 32) & (C - 1)) == 0 || p.tin + e0 + 32 == Fk))
+          row_ptr[row0 + (x0 >> csh) + 1] = uint32_t(tile_off + lpre);
       }
-      if ((full || e < p.te) && (col == C - 1 || p.tin + e + 1 == Fk))
-        row_ptr[row0 + ro + 1] = uint32_t(rank + (v != 0));
-      pre += __popc(b);
+    }
+  } else {
+#pragma unroll 1
+    for (int m0 = 0; m0 < G::ROWS; m0 += B) {
+      T vb[B];
+#pragma unroll
+      for (int u = 0; u < B; u++) {
+        const uint32_t e = warp * G::PER_WARP + 32 * (m0 + u) + lane;
+        vb[u] = (full || e < p.te) ? src[e] : T(0);
+      }
+#pragma unroll
+      for (int u = 0; u < B; u++) {
+        const uint32_t e = warp * G::PER_WARP + 32 * (m0 + u) + lane;
+        const T v = vb[u];
+        const uint32_t b = __ballot_sync(0xffffffffu, v != 0);
+        const uint32_t r = lpre + __popc(b & lt);
+        const uint32_t x = cbase + e;
+        const uint32_t ro = pow2 ? x >> csh : x / C;
+        const uint32_t col = x - ro * C;
+        if (v != 0) {
+          tcol[r] = col;
+          tval[r] = v;
+        }
+        if ((full || e < p.te) && (col == C - 1 || p.tin + e + 1 == Fk))
+          row_ptr[row0 + ro + 1] = uint32_t(tile_off + r + (v != 0));
+        lpre += __popc(b);
+      }
     }
   }
   if (tid == 0 && p.j == 0) row_ptr[0] = 0;
