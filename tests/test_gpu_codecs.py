@@ -139,3 +139,26 @@ def test_lz4_match_offsets(C, gap):
     ctl = O.compress(_lz4_offset_case(gap, False), O.LZ4, O.F32, F=1 << 22, param=65536)
     assert len(ref) + 3 * 50 < len(ctl)
     check_parity(C, x, O.LZ4, O.F32)
+
+
+@pytest.mark.parametrize("dtype", [O.F32, O.F16])
+@pytest.mark.parametrize("F,C_row", [(3072, 1), (3072, 3), (3072, 48), (3072, 1536), (3072, 3072),
+                                     (1 << 16, 32), (1 << 16, 64), (1 << 20, 16384), (1 << 20, 65536),
+                                     (1 << 20, 1 << 20)])
+def test_csr_row_widths(C, dtype, F, C_row):
+    """CSR with every kind of row width the header allows (C divides F): rows shorter than a
+    32-element warp row (C = 1, 3), non-power-of-two C (48, 1536, 3072: general emit path),
+    power-of-two C >= 32 (the emit's fast path), and rows longer than a 32 KiB tile (16384 …
+    F: a tile ends mid-row, the frame end closes the last row)."""
+    n = 2 * F + F // 3 + 5
+    x = synth.relu_iid(n, 0.6, seed=F ^ C_row ^ dtype, dtype=dtype)
+    check_parity(C, x, O.CSR, dtype, F=F, C_row=C_row)
+
+
+@pytest.mark.parametrize("B", [1024, 4096, 16384, 65536])
+@pytest.mark.parametrize("kind", ["iid", "clustered"])
+def test_lz4_block_sizes(C, B, kind):
+    """LZ4 with every block size class the header allows (multiple of 1024, <= 65536)."""
+    n = 3 * 16384 + 123
+    x = synth.relu_iid(n, 0.5, seed=B) if kind == "iid" else synth.relu_clustered(n, 0.8, 64, seed=B)
+    check_parity(C, x, O.LZ4, O.F32, F=1 << 16, B=B)
