@@ -405,6 +405,14 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
   CU(cudaMalloc(&b.sc.tbuf2, tiles * 32));  // 32 B per tile: CSR keeps 8 u32 slab counts
   CU(cudaMalloc(&b.sc.aux3, aux * 8));
   CU(cudaMemset(b.sc.status, 0, tiles * 8));
+  // epoch-tagged words are also polled in aux (frame starts): a fresh block restarts at epoch 0,
+  // so memory recycled from an earlier block could hold words tagged with a live epoch; zero
+  // every scratch array once (compute-sanitizer initcheck flagged the first reads of aux)
+  CU(cudaMemset(b.sc.aux, 0, aux * 8));
+  CU(cudaMemset(b.sc.aux2, 0, aux * 8));
+  CU(cudaMemset(b.sc.aux3, 0, aux * 8));
+  CU(cudaMemset(b.sc.tbuf, 0, tiles * 8));
+  CU(cudaMemset(b.sc.tbuf2, 0, tiles * 32));
   CU(cudaMemset(b.sc.tickets, 0, kEpochs * 4));
   CU(cudaMemset(b.sc.err, 0, 64));
   b.sc.cap_tiles = tiles;

@@ -326,7 +326,10 @@ __global__ void __launch_bounds__(32 * kLz4Warps) lz4_decode_kernel(const uint8_
     if (offset == 0 || offset > op || op + mlen > L) { bad = true; break; }
     __syncwarp();  // the match source may have been written by other lanes
     if (offset >= 32) {  // non-overlapping within a 32-byte step
-      const bool near = offset <= kLz4Ring;  // source still in the ring
+      // source still in the ring, and not in a slot this 32-byte step overwrites (a step writes
+      // positions up to o + 31, i.e. ring slots of positions up to 31 bytes past o - kLz4Ring;
+      // compute-sanitizer racecheck found offsets 4065..4095 racing before this bound)
+      const bool near = offset + 32 <= kLz4Ring;
       for (uint32_t q = 0; q < mlen; q += 32) {
         if (q + lane < mlen) {
           const uint32_t o = op + q + lane;

@@ -346,6 +346,9 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       uint32_t v[B];
 #pragma unroll
       for (int u = 0; u < B; u++) v[u] = load_elem(full_tag, stage, gsrc, e0 + 32 * (m0 + u), te, be);
+      // the batch's compaction stores may overwrite words other lanes just loaded: order every
+      // lane's loads before any lane's stores (a ballot synchronises but does not order memory)
+      __syncwarp();
 #pragma unroll
       for (int u = 0; u < B; u++) {
         const uint32_t w = __ballot_sync(0xffffffffu, v[u] != 0);

@@ -127,7 +127,7 @@ def _lz4_offset_case(gap: int, repeat: bool) -> np.ndarray:
     return x
 
 
-@pytest.mark.parametrize("gap", [3, 31, 32, 33, 4000, 4096, 4097, 10000, 60000])
+@pytest.mark.parametrize("gap", [3, 31, 32, 33, 4000, 4064, 4065, 4070, 4090, 4095, 4096, 4097, 10000, 60000])
 def test_lz4_match_offsets(C, gap):
     """Every match-offset class of the LZ4 decoder: overlapping short offsets (< 32 bytes,
     pattern replication), offsets served by the warp's 4 KiB recent-output ring, and offsets
