@@ -110,6 +110,24 @@ constexpr bool kStaticTiles = true;
 constexpr bool kStaticTiles = false;
 #endif
 
+// store of one 16- or 32-bit word at a shared byte address.  Only the in-place compaction uses
+// it: its stores land at or before the rows already loaded (count_slab), so the compiler may move
+// later loads across it (no "memory" clobber).
+template <typename T>
+__device__ __forceinline__ void sts_word(uint32_t a, uint32_t x) {
+  if constexpr (sizeof(T) == 4) asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(x));
+  else asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"(uint16_t(x)));
+}
+
+// a * W + c, opaque to the front end's reassociation (which would otherwise turn the running
+// byte address back into an element count plus a scaled add per store)
+template <int W>
+__device__ __forceinline__ uint32_t mad_u32(uint32_t a, uint32_t c) {
+  uint32_t r;
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "n"(W), "r"(c));
+  return r;
+}
+
 // compress tile geometry: TB bytes per tile
 template <typename T, int TB>
 struct CGeom {
@@ -340,7 +358,10 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     constexpr int B = EROWS < CSWAP_ZVC_BATCH ? EROWS : CSWAP_ZVC_BATCH;
     const uint32_t e0 = warp * PW + lane;
     T* sv = reinterpret_cast<T*>(stage) + warp * PW;
-    uint32_t tot = 0;
+    // shared byte address of the next compacted slot, so a lane's store address is one shift-add
+    // (an element index costs an add and a scaled add per row)
+    const uint32_t sdp0 = uint32_t(__cvta_generic_to_shared(sv));
+    uint32_t sdp = sdp0;
 #pragma unroll
     for (int m0 = 0; m0 < EROWS; m0 += B) {
       uint32_t v[B];
@@ -353,12 +374,12 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       for (int u = 0; u < B; u++) {
         const uint32_t w = __ballot_sync(0xffffffffu, v[u] != 0);
         if (lane == 0) bm_out[m0 + u] = w;
-        if (v[u]) sv[tot + __popc(w & lt)] = T(v[u]);
-        tot += __popc(w);
+        if (v[u]) sts_word<T>(mad_u32<G::W>(__popc(w & lt), sdp), v[u]);
+        sdp = mad_u32<G::W>(__popc(w), sdp);
       }
     }
     __syncwarp();
-    return tot;
+    return (sdp - sdp0) / G::W;
   };
 
   // copy the slab's compacted non-zeros (count_slab) to the container (emit_words)
