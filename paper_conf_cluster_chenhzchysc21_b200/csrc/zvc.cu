@@ -78,6 +78,9 @@ constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 #endif
 constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
 // rows per batch of count_slab's loads
+#ifndef CSWAP_ZVC_BM4
+#define CSWAP_ZVC_BM4 1
+#endif
 #ifndef CSWAP_ZVC_BATCH
 #define CSWAP_ZVC_BATCH 16
 #endif
@@ -364,7 +367,8 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     uint32_t sdp = sdp0;
 #pragma unroll
     for (int m0 = 0; m0 < EROWS; m0 += B) {
-      uint32_t v[B];
+      uint32_t v[B], wq[4];
+      static_assert(B % 4 == 0, "bitmap words are stored in fours");
 #pragma unroll
       for (int u = 0; u < B; u++) v[u] = load_elem(full_tag, stage, gsrc, e0 + 32 * (m0 + u), te, be);
       // the batch's compaction stores may overwrite words other lanes just loaded: order every
@@ -373,7 +377,14 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
 #pragma unroll
       for (int u = 0; u < B; u++) {
         const uint32_t w = __ballot_sync(0xffffffffu, v[u] != 0);
-        if (lane == 0) bm_out[m0 + u] = w;
+        // bitmap words leave lane 0 four at a time (one 16-byte shared store per 4 rows)
+        if (CSWAP_ZVC_BM4) {
+          wq[u & 3] = w;
+          if ((u & 3) == 3 && lane == 0)
+            *reinterpret_cast<uint4*>(bm_out + m0 + u - 3) = make_uint4(wq[0], wq[1], wq[2], wq[3]);
+        } else if (lane == 0) {
+          bm_out[m0 + u] = w;
+        }
         if (v[u]) sts_word<T>(mad_u32<G::W>(__popc(w & lt), sdp), v[u]);
         sdp = mad_u32<G::W>(__popc(w), sdp);
       }
