@@ -78,11 +78,14 @@ constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 #endif
 constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
 // rows per batch of count_slab's loads
+#ifndef CSWAP_ZVC_PF
+#define CSWAP_ZVC_PF 1
+#endif
 #ifndef CSWAP_ZVC_BM4
 #define CSWAP_ZVC_BM4 1
 #endif
 #ifndef CSWAP_ZVC_BATCH
-#define CSWAP_ZVC_BATCH 16
+#define CSWAP_ZVC_BATCH 4
 #endif
 // mbarrier waits sleep between tests (max ns): the producer refills a stage whose TMA load takes
 // ~1 us anyway; a resolver has LAG tile periods (~1.5 us each) before its offset is needed; the
@@ -357,7 +360,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     // row m = elements [32m, 32m+32) of the slab: one ballot is bitmap word (slab word m); the
     // non-zeros are compacted in place to the start of the slab (a row's writes land at or
     // before the row, and every row of a batch is loaded before any of its writes).
-    // Rows go in batches of 16 so the batch's loads issue back to back.
+    // Rows go in batches of 4 (CSWAP_ZVC_BATCH) so the batch's loads issue back to back.
     constexpr int B = EROWS < CSWAP_ZVC_BATCH ? EROWS : CSWAP_ZVC_BATCH;
     const uint32_t e0 = warp * PW + lane;
     T* sv = reinterpret_cast<T*>(stage) + warp * PW;
@@ -365,15 +368,22 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     // (an element index costs an add and a scaled add per row)
     const uint32_t sdp0 = uint32_t(__cvta_generic_to_shared(sv));
     uint32_t sdp = sdp0;
+    uint32_t v[B], vn[B];
+#pragma unroll
+    for (int u = 0; u < B; u++) v[u] = load_elem(full_tag, stage, gsrc, e0 + 32 * u, te, be);
 #pragma unroll
     for (int m0 = 0; m0 < EROWS; m0 += B) {
-      uint32_t v[B], wq[4];
+      uint32_t wq[4];
       static_assert(B % 4 == 0, "bitmap words are stored in fours");
-#pragma unroll
-      for (int u = 0; u < B; u++) v[u] = load_elem(full_tag, stage, gsrc, e0 + 32 * (m0 + u), te, be);
       // the batch's compaction stores may overwrite words other lanes just loaded: order every
       // lane's loads before any lane's stores (a ballot synchronises but does not order memory)
       __syncwarp();
+      // software pipelining: the next batch's loads issue before this batch's stores (those land
+      // at or before this batch's rows, never in the next batch's)
+      if (CSWAP_ZVC_PF && m0 + B < EROWS) {
+#pragma unroll
+        for (int u = 0; u < B; u++) vn[u] = load_elem(full_tag, stage, gsrc, e0 + 32 * (m0 + B + u), te, be);
+      }
 #pragma unroll
       for (int u = 0; u < B; u++) {
         const uint32_t w = __ballot_sync(0xffffffffu, v[u] != 0);
@@ -387,6 +397,15 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         }
         if (v[u]) sts_word<T>(mad_u32<G::W>(__popc(w & lt), sdp), v[u]);
         sdp = mad_u32<G::W>(__popc(w), sdp);
+      }
+      if (m0 + B < EROWS) {
+        if (!CSWAP_ZVC_PF) {
+          __syncwarp();  // this batch's stores before the next batch's loads
+#pragma unroll
+          for (int u = 0; u < B; u++) vn[u] = load_elem(full_tag, stage, gsrc, e0 + 32 * (m0 + B + u), te, be);
+        }
+#pragma unroll
+        for (int u = 0; u < B; u++) v[u] = vn[u];
       }
     }
     __syncwarp();

@@ -1,10 +1,16 @@
-# Round-end check with the final tree: GPU tests, smoke, bench lines (VGG16 default, ResNet-50,
-# BERT), the torchrun launch path (1 process; NCCL max-over-ranks) and the reference arm.
-set -x
-timeout 1500 python -m pytest tests -q -m gpu 2>&1 | tail -3 > gpurun_out/f_pytest.log
-timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/f_smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/f_smoke.log
+# final-tree check: GPU tests, smoke, bench line, ZVC table, batch-8 A/B
+mkdir -p gpurun_out
+timeout 1500 python -m pytest tests -q -m gpu -x 2>&1 | tail -2
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -1
 timeout 900 python bench.py > gpurun_out/f_bench.json 2> gpurun_out/f_bench.err
-timeout 900 python bench.py --workload resnet50 --no-cpu > gpurun_out/f_bench_resnet.json 2> gpurun_out/f_bench_resnet.err
-timeout 900 python bench.py --workload bert --no-cpu > gpurun_out/f_bench_bert.json 2> gpurun_out/f_bench_bert.err
-timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 1 --master-addr 127.0.0.1 --master-port 29517 bench.py --gpus 1 --steps 3 --warmup 3 --no-extras --no-cpu > gpurun_out/f_torchrun.json 2> gpurun_out/f_torchrun.err
-timeout 900 python bench.py --impl reference --steps 2 --warmup 3 > gpurun_out/f_ref.json 2> gpurun_out/f_ref.err
+python -c "
+import json
+r=json.loads(open('gpurun_out/f_bench.json').read().strip().splitlines()[-1]); x=r['extras']
+print(r['value'], r['ms_per_step'], r['roofline']['frac'], r['roofline']['device_clock']['frac'], r['roofline']['isolated'], x['latency_ms'], x['link'], r['e2e']['value'], r['clocks'])"
+bash tools/run_zvc_table.sh 2>&1 | tail -14
+for v in pf8; do for d in f32 f16; do CSWAP_LIB_VARIANT=$v timeout 300 python tools/codec_bench.py --codecs zvc --mib 1024 --s 0.2,0.5,0.95 --dtype $d 2>&1 | python -c "
+import sys,json
+for l in sys.stdin:
+    try: r=json.loads(l)
+    except Exception: continue
+    print('$v', r['dtype'], r['s'], 'c', r['compress']['ms'], r['compress']['frac'])"; done; done
