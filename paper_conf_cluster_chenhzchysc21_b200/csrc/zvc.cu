@@ -78,6 +78,9 @@ constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 #endif
 constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
 // rows per batch of count_slab's loads
+#ifndef CSWAP_ZVC_POW2
+#define CSWAP_ZVC_POW2 1
+#endif
 #ifndef CSWAP_ZVC_PF
 #define CSWAP_ZVC_PF 1
 #endif
@@ -194,10 +197,12 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
   }
   __syncthreads();
 
+  const bool tpf_pow2 = CSWAP_ZVC_POW2 && (tpf & (tpf - 1)) == 0;
+  const int tpf_sh = __ffs(int(tpf)) - 1;
   auto tile_geom = [&](uint32_t t, uint32_t& k, uint32_t& j, uint64_t& Fk, uint32_t& tile_elems,
                        uint32_t& bulk_elems) {
-    k = t / tpf;
-    j = t % tpf;
+    k = tpf_pow2 ? t >> tpf_sh : t / tpf;  // tiles per frame is a power of two for power-of-two
+    j = tpf_pow2 ? t & (tpf - 1) : t % tpf;  // frames: a shift instead of a ~20-instruction divide
     Fk = frame_len(n, F, k);
     tile_elems = uint32_t(umin64(G::TILE, Fk - uint64_t(j) * G::TILE));
     bulk_elems = ((tile_elems * G::W) & ~15u) / G::W;
@@ -250,7 +255,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       const uint32_t nnz = s_nnz[s];
       if (nnz == SENT) break;
       const uint32_t t = s_ticket[s];
-      const uint32_t k = t / tpf, j = t % tpf;
+      const uint32_t k = tpf_pow2 ? t >> tpf_sh : t / tpf, j = tpf_pow2 ? t & (tpf - 1) : t % tpf;
       const uint64_t nwords_k = cdiv(frame_len(n, F, k), 32);
       uint64_t excl = 0, fstart = 0;
       // offset = frame start + bitmap + W * (totals of earlier 32-tile groups of the frame +

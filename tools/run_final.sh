@@ -1,4 +1,4 @@
-# final-tree check: GPU tests, smoke, bench line, ZVC table, batch-8 A/B
+# final-tree check: GPU tests, smoke, bench line, ZVC table
 mkdir -p gpurun_out
 timeout 1500 python -m pytest tests -q -m gpu -x 2>&1 | tail -2
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -1
@@ -8,9 +8,3 @@ import json
 r=json.loads(open('gpurun_out/f_bench.json').read().strip().splitlines()[-1]); x=r['extras']
 print(r['value'], r['ms_per_step'], r['roofline']['frac'], r['roofline']['device_clock']['frac'], r['roofline']['isolated'], x['latency_ms'], x['link'], r['e2e']['value'], r['clocks'])"
 bash tools/run_zvc_table.sh 2>&1 | tail -14
-for v in pf8; do for d in f32 f16; do CSWAP_LIB_VARIANT=$v timeout 300 python tools/codec_bench.py --codecs zvc --mib 1024 --s 0.2,0.5,0.95 --dtype $d 2>&1 | python -c "
-import sys,json
-for l in sys.stdin:
-    try: r=json.loads(l)
-    except Exception: continue
-    print('$v', r['dtype'], r['s'], 'c', r['compress']['ms'], r['compress']['frac'])"; done; done
