@@ -46,7 +46,9 @@ def test_config1_parity(C, codec):
 @pytest.mark.parametrize("codec", CODECS)
 @pytest.mark.parametrize("dtype", [O.F32, O.F16, O.BF16])
 @pytest.mark.parametrize("n,F", [(1, 1024), (31, 1024), (1000, 1024), (8192, 1024), (8193, 1 << 13),
-                                 (100003, 1 << 14), (250000, 1 << 20), (3 * 16384 + 7, 16384)])
+                                 (100003, 1 << 14), (250000, 1 << 20), (3 * 16384 + 7, 16384),
+                                 # tiles per frame not a power of two (the compress kernel's divide path)
+                                 (300001, 5 * 8192), (200000, 3 * 1024 * 7)])
 def test_ragged_sizes_and_frames(C, codec, dtype, n, F):
     x = synth.relu_iid(n, 0.55, seed=n ^ F ^ dtype, dtype=dtype)
     check_parity(C, x, codec, dtype, F=F)
