@@ -8,8 +8,11 @@ value = raw tensor bytes swapped out and back in per second, summed over ranks (
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
                     [--workload vgg16|resnet50|bert] [--calibrate] [--no-extras]
-Multi-GPU: one process per GPU under torchrun; each rank swaps its own replica of the set
-(no collective on the data path, "scaling": "weak"); time = max over ranks.
+Multi-GPU ("replicas only"): one process per GPU, each swapping its own replica
+of the set (no collective on the data path, "scaling": "weak"); time = the slowest rank's device
+time.  Under torchrun the ranks come from the environment; `python bench.py --gpus N` without
+torchrun starts the N rank processes itself (RANK / LOCAL_RANK / WORLD_SIZE set per child).  The
+ranks meet only on a CPU (gloo) barrier and one MAX / gather of per-rank numbers.
 """
 from __future__ import annotations
 
@@ -145,6 +148,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
         return hs
 
     def barrier():
+        torch.cuda.synchronize()
         if dist is not None:
             dist.barrier()
         torch.cuda.synchronize()
@@ -224,6 +228,16 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
         result["extras"] = _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, raw_bytes,
                                    world)
         result["e2e"] = _e2e(args, C, torch, tensors, outs, sizes, dtype, w, dist, world, stream)
+    # per-rank numbers, measured with every rank running at once (replicas share the host links)
+    rank_info = {"rank": rank, "ms_per_step": round(main["ms"] / args.steps, 4), "host_binding": numa}
+    if "extras" in result:
+        ex = result["extras"]
+        rank_info.update(link=ex["link"], every_compressed_tensor_faster=ex["every_compressed_tensor_faster"],
+                         swap_latency_reduction_vs_vdnn=round(ex["swap_latency_reduction_vs_vdnn"], 4))
+    per_rank = _gather(dist, rank_info)
+    result["per_rank"] = per_rank
+    if "extras" in result:
+        result["every_compressed_tensor_faster_all_ranks"] = all(p["every_compressed_tensor_faster"] for p in per_rank)
     if rank == 0 and world == 1 and not args.no_cpu:
         result["cpu_baseline"] = _cpu_baseline(tensors, sizes, decisions, dtype)
     return result
@@ -250,8 +264,7 @@ def _max_over_ranks(v: float, dist) -> float:
     if dist is None or not dist.is_initialized():
         return v
     import torch
-    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
-    t = torch.tensor([v], dtype=torch.float64, device=dev)
+    t = torch.tensor([v], dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -397,6 +410,9 @@ def _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, r
     """Baselines in the same run: vDNN (NONE), SC (always ZVC), the Orac bound; link GB/s;
     per-tensor latency check (compressed < uncompressed for every tensor the selector compressed)."""
     ex = {}
+    if dist is not None:  # all ranks measure the link at the same time (shared PCIe / host DRAM)
+        torch.cuda.synchronize()
+        dist.barrier()
     link = _link(torch)
     ex["link"] = link
     steps_b = max(2, min(args.steps, 3))
@@ -409,7 +425,11 @@ def _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, r
     ex["latency_ms"]["orac_bound"] = orac * 1e3
     ex["latency_ms"]["raw_link_bound"] = (raw_bytes / (link["d2h_GBps"] * 1e9) + raw_bytes / (link["h2d_GBps"] * 1e9)) * 1e3
     ex["swap_latency_reduction_vs_vdnn"] = 1 - ex["latency_ms"]["auto"] / ex["latency_ms"]["vdnn_none"]
-    # per-tensor: the selector's choice vs NONE, measured one tensor at a time
+    # per-tensor: the selector's choice vs NONE, measured one tensor at a time (on every rank at
+    # once: SURVEY §8(d) asks for compressed < uncompressed with all GPUs swapping concurrently)
+    if dist is not None:
+        torch.cuda.synchronize()
+        dist.barrier()
     per = []
     stream = torch.cuda.current_stream()
     for i, (t, o, n) in enumerate(zip(tensors, outs, sizes)):
@@ -643,7 +663,62 @@ def run_reference(args, rank: int, world: int) -> dict | None:
             "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
 
 
-def main():
+def _free_port() -> int:
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+def spawn_replicas(args, argv) -> int:
+    """`python bench.py --gpus N` outside torchrun: start one rank process per GPU (same argv,
+    RANK / LOCAL_RANK / WORLD_SIZE / MASTER_* in the environment) and wait for all of them.  Rank
+    0 prints the one JSON line (stdout is inherited).  Asking for more GPUs than are visible is an
+    error, never a silent N = 1."""
+    if not args.stub:
+        import torch
+        visible = torch.cuda.device_count()
+        if args.gpus > visible:
+            print(f"bench.py: --gpus {args.gpus} but only {visible} CUDA device(s) are visible", file=sys.stderr)
+            return 2
+    port = _free_port()
+    procs = []
+    for r in range(args.gpus):
+        env = dict(os.environ, RANK=str(r), LOCAL_RANK=str(r), WORLD_SIZE=str(args.gpus),
+                   LOCAL_WORLD_SIZE=str(args.gpus), MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        procs.append(subprocess.Popen([sys.executable, os.path.abspath(__file__), *argv], env=env))
+    rcs = [p.wait() for p in procs]
+    return max(rcs, key=abs)
+
+
+def run_stub(args, rank: int, world: int, dist) -> dict | None:
+    """CPU-only stand-in for run_ours (tests/test_multirank_cpu.py): exercises the launcher, the
+    CPU barrier and the aggregation with a fake per-rank device time (rank r: 10 (r + 1) ms per
+    step) and 1 MiB of 'swapped' bytes per rank."""
+    raw = 1 << 20
+    ms_rank = 10.0 * (rank + 1)
+    if dist is not None:
+        dist.barrier()
+    ms_max = _max_over_ranks(ms_rank * args.steps, dist) / args.steps
+    per_rank = _gather(dist, {"rank": rank, "ms_per_step": ms_rank, "pid": os.getpid(),
+                              "every_compressed_tensor_faster": True})
+    return {"metric": METRIC, "value": round(job_throughput(world, raw, ms_max), 6), "unit": "GB/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max,
+            "higher_is_better": True, "scaling": "weak", "data": "stub", "per_rank": per_rank,
+            "every_compressed_tensor_faster_all_ranks": all(p["every_compressed_tensor_faster"] for p in per_rank)}
+
+
+def _gather(dist, obj) -> list:
+    """Every rank's `obj`, in rank order (rank 0 alone: [obj])."""
+    if dist is None or not dist.is_initialized():
+        return [obj]
+    out = [None] * dist.get_world_size()
+    dist.all_gather_object(out, obj)
+    return out
+
+
+def main(argv=None):
+    argv = sys.argv[1:] if argv is None else argv
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
@@ -653,9 +728,16 @@ def main():
     ap.add_argument("--calibrate", action="store_true", help="full calibration sweep, writes calib/b200.json")
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    args = ap.parse_args()
+    ap.add_argument("--stub", action="store_true", help=argparse.SUPPRESS)  # CPU test of the launcher
+    args = ap.parse_args(argv)
     if args.warmup < 3:
         args.warmup = 3
+    if args.gpus < 1:
+        print("bench.py: --gpus must be >= 1", file=sys.stderr)
+        return 2
+    under_launcher = "WORLD_SIZE" in os.environ
+    if not under_launcher and args.gpus > 1 and args.impl == "ours":
+        return spawn_replicas(args, argv)
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
@@ -663,20 +745,25 @@ def main():
         res = run_reference(args, rank, world)
         if res is not None:
             print(json.dumps(res), flush=True)
-        return
+        return 0
+    if world != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but the launcher started {world} rank(s)", file=sys.stderr)
+        return 2
     dist = None
     if world > 1:
-        import torch
         import torch.distributed as tdist
-        torch.cuda.set_device(local_rank)
-        tdist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        # replicas only: a CPU (gloo) group for the barrier and the MAX / gather of per-rank
+        # numbers; nothing on the data path crosses GPUs (no NCCL)
+        tdist.init_process_group("gloo")
         dist = tdist
-    res = run_ours(args, rank, world, local_rank, dist)
+    res = run_stub(args, rank, world, dist) if args.stub else run_ours(args, rank, world, local_rank, dist)
     if rank == 0 and res is not None:
         print(json.dumps(res), flush=True)
     if dist is not None:
+        dist.barrier()
         dist.destroy_process_group()
+    return 0
 
 
 if __name__ == "__main__":
-    main()
+    sys.exit(main())

@@ -59,3 +59,42 @@ def test_job_throughput_counts_all_ranks():
     eight = bench.job_throughput(8, raw, 46.4)
     assert eight == pytest.approx(8 * one)
     assert one == pytest.approx(raw / 0.0464 / 1e9)
+
+
+def _run_bench(args, env_extra=None, timeout=240):
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = {k: v for k, v in os.environ.items() if k not in ("RANK", "LOCAL_RANK", "WORLD_SIZE", "MASTER_ADDR",
+                                                            "MASTER_PORT", "LOCAL_WORLD_SIZE")}
+    env.update(env_extra or {})
+    p = subprocess.run([sys.executable, os.path.join(root, "bench.py"), *args], capture_output=True, text=True,
+                       timeout=timeout, env=env, cwd=root)
+    lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+    return p.returncode, [json.loads(ln) for ln in lines], p.stderr
+
+
+def test_bench_gpus_n_spawns_n_replicas_stub():
+    """`python bench.py --gpus 2` (no torchrun) starts two rank processes itself; they meet on a
+    gloo barrier, rank 0 prints ONE line with n_gpus = 2, the job time is the slowest rank's and
+    the throughput counts both ranks' bytes (stub workload: rank r takes 10 (r + 1) ms/step)."""
+    rc, out, err = _run_bench(["--gpus", "2", "--stub", "--steps", "2", "--warmup", "3"])
+    assert rc == 0, err
+    assert len(out) == 1
+    res = out[0]
+    assert res["n_gpus"] == 2 and res["scaling"] == "weak"
+    assert [p["rank"] for p in res["per_rank"]] == [0, 1]
+    assert len({p["pid"] for p in res["per_rank"]}) == 2  # two processes
+    assert res["ms_per_step"] == pytest.approx(20.0)
+    assert res["value"] == pytest.approx(2 * (1 << 20) / 0.020 / 1e9, rel=1e-5)
+    assert res["every_compressed_tensor_faster_all_ranks"] is True
+
+
+def test_bench_rejects_gpu_count_mismatch():
+    # under a launcher that started 2 ranks, --gpus 3 is an error (never a silent other N)
+    rc, out, err = _run_bench(["--gpus", "3", "--stub"], {"WORLD_SIZE": "2", "RANK": "0", "LOCAL_RANK": "0"})
+    assert rc == 2 and not out and "launcher started 2" in err
+    # more GPUs than visible (none on this CPU box) is an error too
+    rc, out, err = _run_bench(["--gpus", "4", "--no-extras"], timeout=120)
+    assert rc == 2 and not out and "visible" in err
