@@ -593,26 +593,109 @@ def _e2e(args, C, torch, tensors, outs, sizes, dtype, w, dist, world, stream) ->
             "h2d_bytes_per_step": raw, "d2h_bytes_per_step": 16 * len(tensors), "steps": steps}
 
 
-def _cpu_baseline(tensors, sizes, decisions, dtype, sample_mib=16) -> dict:
-    """The plain-C oracle, as it stands, on the host cores: per tensor the first `sample_mib` MiB
-    are compressed and decompressed with the codec the selector chose (NONE = raw copy)."""
-    import numpy as np
+def _cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
+def _oracle_seconds(xs, codec: int, dtype: int, threads: int) -> float:
+    """Seconds for the plain-C oracle, as it stands, to compress and then decompress every
+    array of `xs` with `codec`, frame by frame (F = 2^22 elements, the container default).
+    With threads > 1 the frames of all arrays are spread over a pool of host threads (the
+    ctypes call releases the GIL, so each thread runs the scalar C code on its own frames: the
+    "OpenMP over frames, timing only" of SURVEY §8(d)); the oracle itself is unchanged."""
+    import concurrent.futures as cf
+
     from oracle import oracle as O
+    F = O.DEFAULT_F
+    frames = [x[k:k + F] for x in xs for k in range(0, x.size, F)]
+
+    def one(fr):
+        blob = O.compress(fr, codec, dtype)
+        O.decompress(blob, fr.size, dtype)
+
+    t0 = time.perf_counter()
+    if threads <= 1:
+        for fr in frames:
+            one(fr)
+    else:
+        with cf.ThreadPoolExecutor(max_workers=threads) as ex:
+            list(ex.map(one, frames))
+    return time.perf_counter() - t0
+
+
+def _cpu_baseline(tensors, sizes, decisions, dtype) -> dict:
+    """The plain-C oracle on the host cores (SURVEY §8(d) "oracle timing"; PAPER.md:251 compares
+    with vDNN++'s 64 CPU threads): compress + decompress with the codec the selector chose for
+    each tensor (NONE = raw copy), on a bounded sample of every tensor of the set.  `value` = all
+    host cores (frames spread over threads), `single_thread` on a smaller sample."""
+    import numpy as np
     w = 4 if dtype == 0 else 2
-    tot_bytes, tot_s = 0, 0.0
-    for t, n, codec in zip(tensors, sizes, decisions):
-        m = min(n, sample_mib * 2**20 // w)
-        x = t[:m].cpu().numpy()
-        x = x.view(np.uint32) if w == 4 else x.view(np.uint16)
-        t0 = time.perf_counter()
-        blob = O.compress(x, codec, dtype)
-        y = O.decompress(blob, m, dtype)
-        tot_s += time.perf_counter() - t0
-        assert np.array_equal(x, y)
-        tot_bytes += m * w
-    return {"value": round(tot_bytes / tot_s / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"first {sample_mib} MiB of each of the {len(sizes)} tensors ({tot_bytes / 2**20:.0f} MiB), "
-                      f"oracle compress+decompress with the selector's codec, single thread, {tot_s:.1f} s"}
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+
+    def sample(mib):
+        xs, tot = [], 0
+        for t, n in zip(tensors, sizes):
+            m = min(n, mib * 2**20 // w)
+            x = t[:m].cpu().numpy()
+            xs.append(x.view(np.uint32) if w == 4 else x.view(np.uint16))
+            tot += m * w
+        return xs, tot
+
+    def timed(xs, threads):
+        secs = 0.0
+        by_codec = {}
+        for x, c in zip(xs, decisions):
+            by_codec.setdefault(c, []).append(x)
+        for c, group in by_codec.items():
+            secs += _oracle_seconds(group, c, dtype, threads)
+        return secs
+
+    xs1, b1 = sample(16)
+    s1 = timed(xs1, 1)
+    xsn, bn = sample(64)
+    sn = timed(xsn, cores)
+    return {"value": round(bn / sn / 1e9, 4), "unit": "GB/s", "cores": cores, "kind": "oracle",
+            "sample": f"first 64 MiB of each of the {len(sizes)} tensors ({bn / 2**20:.0f} MiB), oracle compress+"
+                      f"decompress with the selector's codec, frames spread over {cores} threads, {sn:.1f} s",
+            "single_thread": {"value": round(b1 / s1 / 1e9, 4), "cores": 1,
+                              "sample": f"first 16 MiB of each tensor ({b1 / 2**20:.0f} MiB), {s1:.1f} s"},
+            "cpu_model": _cpu_model(), "cpu_count": os.cpu_count()}
+
+
+def cpu_plan(path: str) -> dict:
+    """SURVEY §8(d) oracle-timing plan (`bench.py --cpu-plan OUT.json`, CPU only): per codec,
+    single thread on config 1 and on the config-2 iid fp32 points up to 64 MiB at s = 0.2 / 0.5 /
+    0.8 and 1 GiB at the same sparsities; all host cores for the points >= 16 MiB."""
+    import synth
+    cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+    rows = []
+    cfg1 = synth.relu_iid(1 << 20, 0.5, seed=synth.seed_of(1), exact=True)
+    points = [("config1_4MiB", cfg1, 0.5)]
+    for si, s in enumerate((0.2, 0.5, 0.8)):
+        for zi, mib in enumerate((0.0625, 0.25, 1, 4, 16, 64, 1024)):
+            n = int(mib * 2**18)
+            points.append((f"iid_{mib}MiB", synth.relu_iid(n, s, seed=synth.seed_of(2, zi, si)), s))
+    for name, x, s in points:
+        for codec in (1, 2, 3, 4):
+            for threads in ((1, cores) if x.nbytes >= 16 << 20 else (1,)):
+                secs = _oracle_seconds([x], codec, 0, threads)
+                rows.append({"point": name, "sparsity": s, "MiB": x.nbytes / 2**20, "codec": codec,
+                             "threads": threads, "s": round(secs, 4), "GBps": round(x.nbytes / secs / 1e9, 4)})
+                log(json.dumps(rows[-1]))
+    out = {"cpu_model": _cpu_model(), "cpu_count": os.cpu_count(), "threads_all": cores,
+           "how": "oracle compress + decompress per frame (F = 2^22), scalar C -O2; threads > 1 spread frames "
+                  "over a host thread pool", "rows": rows}
+    with open(path, "w") as f:
+        json.dump(out, f, indent=1)
+    return out
 
 
 # ------------------------------------------------------------------------------------ reference arm
@@ -729,7 +812,11 @@ def main(argv=None):
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--stub", action="store_true", help=argparse.SUPPRESS)  # CPU test of the launcher
+    ap.add_argument("--cpu-plan", metavar="OUT_JSON", help="oracle timing plan of SURVEY §8(d) (CPU only)")
     args = ap.parse_args(argv)
+    if args.cpu_plan:
+        cpu_plan(args.cpu_plan)
+        return 0
     if args.warmup < 3:
         args.warmup = 3
     if args.gpus < 1:
