@@ -1,15 +1,20 @@
-// api.cu — the C ABI of include/cswap.h: runtime (streams, scratch, pools, handles), codec
-// dispatch, probe + selector, and the swap-out / swap-in pipelines.
+// api.cu — the C ABI of include/cswap.h: runtime (streams, scratch, pools, handles, the swap-out
+// executor thread), codec dispatch, probe + selector, and the swap-out / swap-in pipelines.
 //
 // Swapping executor (PAPER.md:120 §IV-A; :228 §V): compress -> offload to pinned host memory on
 // an asynchronous copy stream; prefetch -> decompress.  Memory pools replace cudaMalloc /
-// cudaMallocHost on the path: device staging comes from the CUDA stream-ordered
-// pool (cudaMallocAsync, release threshold = unlimited), host containers from a pinned-chunk
-// allocator.  Swap-in is pipelined per frame group (R7): H2D of group g+1 overlaps the
-// decompression of group g.
+// cudaMallocHost on the path: device staging comes from a private stream-ordered
+// pool, host containers from a pinned-chunk allocator.  Both directions are pipelined per frame
+// (R7): swap-out hands each frame to the copy engine as soon as the compress kernel
+// publishes it (a library thread issues the D2H copies; the caller never blocks), swap-in's H2D
+// of frame k+1 overlaps the decompression of frame k.
 #include <algorithm>
 #include <atomic>
+#include <chrono>
+#include <condition_variable>
 #include <cstdarg>
+#include <deque>
+#include <thread>
 #include <cstdio>
 #include <cstring>
 #include <map>
@@ -145,7 +150,7 @@ struct PinnedPool {
 };
 
 // ---------------------------------------------------------------------------------------------
-// scratch blocks (lookback status, tickets, per-frame arrays) leased per operation
+// scratch blocks (tile status words, tickets, per-frame arrays) leased per operation
 // ---------------------------------------------------------------------------------------------
 struct Block {
   Scratch sc{};
@@ -156,12 +161,26 @@ struct Block {
 
 constexpr int kBlocks = 4;
 
+struct OutJob;
+
 struct Ctx {
   int device = -1;
   int sms = 0;
   Block blocks[kBlocks];
   std::atomic<uint32_t> rr{0};
-  cudaStream_t s_d2h = nullptr, s_h2d = nullptr;
+  // D2H copy stream; two H2D copy streams that swap-in frames alternate between (an event record
+  // on a copy stream stalls that stream ~25-35 us while PCIe is busy, tools/event_probe.cu: the
+  // other stream's copy keeps the link busy meanwhile)
+  cudaStream_t s_d2h = nullptr, s_h2d = nullptr, s_h2d2 = nullptr;
+  cudaMemPool_t pool = nullptr;  // private stream-ordered pool (staging, LZ4 slots, decode scratch)
+  uint64_t* dev_sink = nullptr;  // device word for container sizes nobody reads
+  // swap-out executor: one library thread turns published frames into D2H copies, FIFO
+  std::thread exec;
+  std::mutex qm;
+  std::condition_variable qcv;
+  std::deque<OutJob*> q;
+  bool stop = false;
+
   std::mutex cfg_m;
   cswap_calib calib{};
   cswap_format fmt{};
@@ -176,7 +195,7 @@ struct Ctx {
   struct Pend {
     cudaEvent_t a, b;
     cswap_kernel_record r;
-    uint64_t* stamps;  // 2 x u64 %globaltimer (mapped pinned), or null
+    uint64_t* stamps;  // 2 x u64 %globaltimer + the container size (mapped pinned), or null
   };
   std::vector<Pend> pend;
 };
@@ -191,7 +210,9 @@ struct Timer {
   cudaStream_t st;
   cudaEvent_t a = nullptr, b = nullptr;
   bool started = false;
-  uint64_t* stamps = nullptr;  // filled by stamp kernels first / last in the group (run_group)
+  // [0], [1]: filled by stamp kernels first / last in the group (run_group); [2]: a swap-out's
+  // compress writes its container size here (read at collection time)
+  uint64_t* stamps = nullptr;
   Timer(Ctx* ctx, cudaStream_t s);
   void start_now() {
     if (a && !started) {
@@ -220,8 +241,8 @@ namespace {
 Timer::Timer(Ctx* ctx, cudaStream_t s) : c(ctx), st(s) {
   if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) {
     t_pending = this;
-    stamps = reinterpret_cast<uint64_t*>(c->pinned.alloc(16));
-    if (stamps) stamps[0] = stamps[1] = 0;
+    stamps = reinterpret_cast<uint64_t*>(c->pinned.alloc(24));
+    if (stamps) stamps[0] = stamps[1] = stamps[2] = 0;
   }
 }
 Timer::~Timer() {
@@ -527,11 +548,25 @@ cswap_status cuda_status(cudaError_t e, const char* what) {
 }
 
 // ---- compress (device -> device or mapped) ---------------------------------------------------
+// prog (swap-out only): host-mapped progress words, see Scratch::prog.  ZVC publishes each frame
+// from inside its persistent kernel; the multi-pass codecs publish every frame once their last
+// kernel has run (a publish kernel at the end of the same launch group).
 cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int codec, const cswap_format& f,
-                         uint8_t* out, uint64_t* out_size, cudaStream_t st) {
+                         uint8_t* out, uint64_t* out_size, cudaStream_t st, uint64_t* prog = nullptr,
+                         bool frame_publish = false) {
   const int w = width(dtype);
   const uint64_t F = f.frame_elems;
   const uint32_t K = uint32_t((n + F - 1) / F);
+  auto publish = [&](cudaStream_t gs) -> cswap_status {
+    if (!prog) return CSWAP_OK;
+    c->launches++;
+    return cuda_status(launch_publish_frames(out, K, prog, gs), "publish_frames");
+  };
+  auto with_prog = [&](const Scratch& sc) {
+    Scratch s2 = sc;
+    s2.prog = prog;
+    return s2;
+  };
   if (n == 0) {
     c->launches++;
     return cuda_status(launch_header_only(out, codec, dtype, F, param_of(codec, f), out_size, st), "header");
@@ -539,7 +574,8 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
   switch (codec) {
     case CSWAP_CODEC_NONE:
       c->launches++;
-      return cuda_status(launch_none_compress(in, n, w, F, dtype, out, out_size, st), "none_compress");
+      TRY(cuda_status(launch_none_compress(in, n, w, F, dtype, out, out_size, st), "none_compress"));
+      return publish(st);
     case CSWAP_CODEC_ZVC: {
       uint64_t tiles = 0, aux = 0;
       zvc_compress_scratch(n, w, F, &tiles, &aux);
@@ -547,8 +583,16 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       TRY(L.status);
       c->launches += 2;  // accumulator zero fill + persistent compress
       const uint32_t ep = L.epoch();
-      return run_group(c, st, group_key(kGrpCompress, codec, dtype), [&](cudaStream_t gs) {
-        return cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, L.b->sc, ep, dtype, gs), "zvc_compress");
+      // per-frame publication from inside the persistent kernel only when asked (the D2H link
+      // is idle, so the first frames' copies can overlap the rest of the compression); it costs
+      // the kernel ~14 us (a gpu-scope acq_rel atomic per tile in the producer warp), so a
+      // swap-out queued behind other copies publishes after the kernel instead
+      const bool inkernel = prog && frame_publish;
+      return run_group(c, st, group_key(kGrpCompress, codec, dtype) | (inkernel ? 1u << 21 : 0u), [&](cudaStream_t gs) {
+        TRY(cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, inkernel ? with_prog(L.b->sc) : L.b->sc, ep,
+                                            dtype, gs),
+                        "zvc_compress"));
+        return inkernel ? CSWAP_OK : publish(gs);
       });
     }
     case CSWAP_CODEC_RLE: {
@@ -557,7 +601,8 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       c->launches += 4;
       const uint32_t ep = L.epoch();
       return run_group(c, st, group_key(kGrpCompress, codec, dtype), [&](cudaStream_t gs) {
-        return cuda_status(launch_rle_compress(in, n, w, F, out, out_size, L.b->sc, ep, dtype, gs), "rle_compress");
+        TRY(cuda_status(launch_rle_compress(in, n, w, F, out, out_size, L.b->sc, ep, dtype, gs), "rle_compress"));
+        return publish(gs);
       });
     }
     case CSWAP_CODEC_CSR: {
@@ -566,14 +611,15 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       c->launches += 4;
       const uint32_t ep = L.epoch();
       return run_group(c, st, group_key(kGrpCompress, codec, dtype), [&](cudaStream_t gs) {
-        return cuda_status(launch_csr_compress(in, n, w, F, f.csr_row, out, out_size, L.b->sc, ep, dtype, gs),
-                           "csr_compress");
+        TRY(cuda_status(launch_csr_compress(in, n, w, F, f.csr_row, out, out_size, L.b->sc, ep, dtype, gs),
+                        "csr_compress"));
+        return publish(gs);
       });
     }
     case CSWAP_CODEC_LZ4: {
       const uint64_t blocks = lz4_scratch_bytes(n, w, F, f.lz4_block);
       uint8_t* slots = nullptr;
-      CU(cudaMallocAsync(&slots, blocks, st));
+      CU(cudaMallocFromPoolAsync(reinterpret_cast<void**>(&slots), blocks, c->pool, st));
       const uint64_t bidx = uint64_t(K) * ((F * w + f.lz4_block - 1) / f.lz4_block);  // block index k*bpf + b
       cswap_status s;
       {
@@ -581,8 +627,9 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
         TRY(L.status);
         c->launches += 3;
         s = run_group(c, st, group_key(kGrpCompress, codec, dtype), [&](cudaStream_t gs) {
-          return cuda_status(launch_lz4_compress(in, n, w, F, f.lz4_block, out, out_size, slots, L.b->sc, dtype, gs),
-                             "lz4_compress");
+          TRY(cuda_status(launch_lz4_compress(in, n, w, F, f.lz4_block, out, out_size, slots, L.b->sc, dtype, gs),
+                          "lz4_compress"));
+          return publish(gs);
         });
       }
       CU(cudaFreeAsync(slots, st));
@@ -650,18 +697,213 @@ cswap_status check_common(const void* p, const char* what) {
 // =============================================================================================
 struct cswap_handle {
   Ctx* ctx = nullptr;
-  uint8_t* host = nullptr;  // container (pinned pool)
-  uint64_t bytes = 0;       // container bytes
+  uint8_t* host = nullptr;  // container (pinned pool): allocated at the codec's worst case, trimmed
+  uint64_t bytes = 0;       // container bytes (valid once out_state != 0)
+  uint64_t cap = 0;         // bytes allocated at `host`
   uint64_t n = 0;
   int dtype = 0, codec = 0;
   cswap_format fmt{};
   cswap_decision dec{};
   cudaEvent_t ev_out = nullptr, ev_in = nullptr;
   bool in_issued = false;
-  uint8_t* slots = nullptr;  // pinned small slots: [0..8) size, [8..12) err
-  uint64_t* size_slot() { return reinterpret_cast<uint64_t*>(slots); }
+  uint8_t* slots = nullptr;  // pinned small slots: [64..68) swap-in error word
   uint32_t* err_slot() { return reinterpret_cast<uint32_t*>(slots + 64); }
+  // swap-out state: 0 = the executor is still issuing the D2H copies, 1 = every copy is issued
+  // and ev_out is recorded on the D2H stream, 2 = failed (out_err / out_msg)
+  std::atomic<int> out_state{0};
+  cswap_status out_err = CSWAP_OK;
+  std::string out_msg;
+  std::mutex m;
+  std::condition_variable cv;
+  // end offset of every frame in the container, as published by the compress kernels (the
+  // executor's copy ranges; swap-in splits its H2D by these trusted values, never by the
+  // host-resident frame table)
+  std::vector<uint64_t> ends;
 };
+
+namespace {
+
+struct OutJob {
+  cswap_handle* h;
+  uint8_t* staging;  // device container written by the compress group
+  uint64_t* prog;    // host-mapped progress words (Scratch::prog)
+  uint32_t K;
+  cudaEvent_t done;  // recorded on the caller's stream after the compress group
+};
+
+void finish_out(cswap_handle* h, int state, cswap_status err, const std::string& msg) {
+  {
+    std::lock_guard<std::mutex> lk(h->m);
+    h->out_err = err;
+    h->out_msg = msg;
+    h->out_state.store(state);
+  }
+  h->cv.notify_all();
+}
+
+// Block until the executor has issued every D2H copy of h (or failed).
+cswap_status wait_out(cswap_handle* h) {
+  if (h->out_state.load() == 0) {
+    std::unique_lock<std::mutex> lk(h->m);
+    h->cv.wait(lk, [&] { return h->out_state.load() != 0; });
+  }
+  if (h->out_state.load() == 2) return fail(h->out_err, "swap-out failed: %s", h->out_msg.c_str());
+  return CSWAP_OK;
+}
+
+// Header + frame table of h's container, written on the host from the frame
+// ends: byte-identical to what the codec kernels write into the device container (the tests
+// compare the whole host container with the oracle), and it saves one small D2H per swap.
+void write_host_header(cswap_handle* h) {
+  const uint64_t F = h->fmt.frame_elems, n = h->n;
+  const uint32_t K = uint32_t((n + F - 1) / F);
+  const uint64_t ds = al16(64 + 8ull * K), total = K ? h->ends.back() : ds;
+  std::memset(h->host, 0, ds);
+  std::memcpy(h->host, "CSWP", 4);
+  const uint16_t ver = 1;
+  std::memcpy(h->host + 4, &ver, 2);
+  h->host[6] = uint8_t(h->codec);
+  h->host[7] = uint8_t(h->dtype);
+  const uint32_t param = param_of(h->codec, h->fmt);
+  std::memcpy(h->host + 8, &n, 8);
+  std::memcpy(h->host + 16, &F, 8);
+  std::memcpy(h->host + 24, &K, 4);
+  std::memcpy(h->host + 28, &param, 4);
+  std::memcpy(h->host + 32, &total, 8);
+  uint64_t prev = ds;
+  for (uint32_t k = 0; k < K; k++) {
+    const uint64_t fb = h->ends[k] - prev;
+    std::memcpy(h->host + 64 + 8ull * k, &fb, 8);
+    prev = h->ends[k];
+  }
+}
+
+// The executor's work for one swap-out: poll the progress words the compress group publishes
+// into host-mapped memory and hand each newly completed run of frames to the copy engine
+// (frame k's D2H overlaps the compression of frames k+1..), then the header + frame table, then
+// record ev_out.  No event is recorded between the frame copies (each record would stall the
+// D2H stream ~30 us behind the link's write queue, tools/event_probe.cu).
+// pipeline granularities (bytes): environment override (read per call, for the A/B probes) or
+// the default of 32 MiB
+uint64_t env_bytes(const char* name, uint64_t dflt) {
+  const char* e = getenv(name);
+  return e ? uint64_t(atof(e) * double(1 << 20)) : dflt;
+}
+
+void run_out_job(Ctx* c, OutJob* j) {
+  cswap_handle* h = j->h;
+  const uint64_t min_copy = env_bytes("CSWAP_COPY_MB", uint64_t(32) << 20);  // D2H copy granularity
+  const uint64_t ds = al16(64 + 8ull * j->K);
+  uint64_t pos = ds;
+  uint32_t k = 0;
+  int idle = 0;
+  bool group_done = false;
+  cswap_status err = CSWAP_OK;
+  std::string msg;
+  h->ends.clear();
+  h->ends.reserve(j->K);
+  const volatile uint64_t* prog = j->prog;
+  uint32_t k_ready = 0;  // frames whose end offset is known (h->ends[0 .. k_ready))
+  while (k < j->K) {
+    while (k_ready < j->K) {
+      const uint64_t v = prog[k_ready];
+      if (!(v & kProgReady)) break;
+      const uint64_t e = v & ~kProgReady;
+      if (e < (k_ready ? h->ends.back() : ds) || e > h->cap || (e & 15)) {
+        err = CSWAP_ERR_CUDA;
+        msg = "inconsistent progress word from the compress kernel";
+        break;
+      }
+      h->ends.push_back(e);
+      k_ready++;
+    }
+    if (err != CSWAP_OK) break;
+    if (k_ready > k) {
+      const uint64_t end = h->ends[k_ready - 1];
+      // copy granularity: a D2H copy costs a few us of DMA ramp and tail (8 MiB copies ran at
+      // 52.2 GB/s, whole tensors at 54.0, tools/pipeline_probe.py), so published frames are
+      // coalesced until `min_copy` bytes are ready -- unless the D2H stream is idle (then any
+      // frame goes at once: this is what overlaps a tensor's first frames with its compression)
+      // or every frame is published
+      if (k_ready < j->K && end - pos < min_copy && cudaStreamQuery(c->s_d2h) == cudaErrorNotReady) {
+        std::this_thread::yield();
+        continue;
+      }
+      if (end > pos &&
+          cudaMemcpyAsync(h->host + pos, j->staging + pos, end - pos, cudaMemcpyDeviceToHost, c->s_d2h) != cudaSuccess) {
+        err = CSWAP_ERR_CUDA;
+        msg = cudaGetErrorString(cudaGetLastError());
+        break;
+      }
+      pos = end;
+      k = k_ready;
+      idle = 0;
+      continue;
+    }
+    if (group_done) {  // the group finished (its writes to mapped memory are visible) but not all frames
+      err = CSWAP_ERR_CUDA;
+      msg = "compress finished without publishing every frame";
+      break;
+    }
+    const cudaError_t e = cudaEventQuery(j->done);
+    if (e == cudaSuccess) {
+      group_done = true;  // one more pass over the progress words
+      continue;
+    }
+    if (e != cudaErrorNotReady) {
+      err = CSWAP_ERR_CUDA;
+      msg = cudaGetErrorString(e);
+      break;
+    }
+    // nothing new yet: spin briefly (a frame completes every few us while the kernel runs),
+    // then back off so that a long queue of pending compresses does not burn a core
+    if (++idle < 4096) std::this_thread::yield();
+    else std::this_thread::sleep_for(std::chrono::microseconds(20));
+  }
+  if (err == CSWAP_OK) write_host_header(h);
+  // staging is freed on the D2H stream behind the copies; when nothing waited for the kernels
+  // (a failure, or n = 0 with no frame to publish) the free is ordered behind the group itself
+  if (err != CSWAP_OK || j->K == 0) cudaStreamWaitEvent(c->s_d2h, j->done, 0);
+  cudaFreeAsync(j->staging, c->s_d2h);
+  cudaEventRecord(h->ev_out, c->s_d2h);
+  cudaEventDestroy(j->done);
+  c->pinned.free(reinterpret_cast<uint8_t*>(j->prog));  // the kernel has written its last word
+  if (err == CSWAP_OK) {
+    h->bytes = pos;
+    c->pinned.shrink(h->host, pos);
+    h->cap = pos;
+  }
+  finish_out(h, err == CSWAP_OK ? 1 : 2, err, msg);
+}
+
+void executor_main(Ctx* c) {
+  cudaSetDevice(c->device);
+  for (;;) {
+    OutJob* j = nullptr;
+    {
+      std::unique_lock<std::mutex> lk(c->qm);
+      c->qcv.wait(lk, [&] { return c->stop || !c->q.empty(); });
+      if (c->q.empty()) return;  // stop requested and drained
+      j = c->q.front();
+    }
+    run_out_job(c, j);
+    {
+      std::lock_guard<std::mutex> lk(c->qm);
+      c->q.pop_front();
+    }
+    delete j;
+  }
+}
+
+void enqueue_out(Ctx* c, OutJob* j) {
+  {
+    std::lock_guard<std::mutex> lk(c->qm);
+    c->q.push_back(j);
+  }
+  c->qcv.notify_one();
+}
+
+}  // namespace
 
 // =============================================================================================
 // C ABI
@@ -704,19 +946,29 @@ cswap_status cswap_init(int device) {
   CU(cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device));
   CU(cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking));
   CU(cudaStreamCreateWithFlags(&c->s_h2d, cudaStreamNonBlocking));
+  CU(cudaStreamCreateWithFlags(&c->s_h2d2, cudaStreamNonBlocking));
   for (auto& b : c->blocks) {
     CU(cudaEventCreateWithFlags(&b.ev, cudaEventDisableTiming));
     TRY(ensure_block(b, 1 << 16, 1 << 12));
   }
-  cudaMemPool_t pool;
-  CU(cudaDeviceGetDefaultMemPool(&pool, device));
-  uint64_t thr = UINT64_MAX;
-  CU(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+  // a private pool ("memory pool"): staging memory stays reserved between swaps up
+  // to a bounded threshold (CSWAP_POOL_KEEP_MB, default 4096) and the process's default pool is
+  // left as the application configured it
+  cudaMemPoolProps pp = {};
+  pp.allocType = cudaMemAllocationTypePinned;
+  pp.location.type = cudaMemLocationTypeDevice;
+  pp.location.id = device;
+  CU(cudaMemPoolCreate(&c->pool, &pp));
+  uint64_t keep = uint64_t(4096) << 20;
+  if (const char* e = getenv("CSWAP_POOL_KEEP_MB")) keep = uint64_t(atoll(e)) << 20;
+  CU(cudaMemPoolSetAttribute(c->pool, cudaMemPoolAttrReleaseThreshold, &keep));
   CU(cudaMalloc(&c->dev_err, 64));
   CU(cudaMemset(c->dev_err, 0, 64));
+  CU(cudaMalloc(&c->dev_sink, 64));
   if (const char* e = getenv("CSWAP_PINNED_CHUNK_MB")) c->pinned.chunk_bytes = uint64_t(atoll(e)) << 20;
   c->calib = builtin_calib();
   c->fmt = cswap_format{uint64_t(1) << 22, 1024, 65536};
+  c->exec = std::thread(executor_main, c);
   g_ctx = c;
   return CSWAP_OK;
 }
@@ -725,6 +977,12 @@ cswap_status cswap_shutdown(void) {
   std::lock_guard<std::mutex> lk(g_mu);
   if (!g_ctx) return CSWAP_OK;
   Ctx* c = g_ctx;
+  {
+    std::lock_guard<std::mutex> lk(c->qm);
+    c->stop = true;
+  }
+  c->qcv.notify_all();
+  if (c->exec.joinable()) c->exec.join();  // drains the queued swap-outs first
   cudaDeviceSynchronize();
   for (auto& b : c->blocks) {
     cudaFree(b.sc.status);
@@ -738,8 +996,11 @@ cswap_status cswap_shutdown(void) {
     cudaEventDestroy(b.ev);
   }
   cudaFree(c->dev_err);
+  cudaFree(c->dev_sink);
+  cudaMemPoolDestroy(c->pool);
   cudaStreamDestroy(c->s_d2h);
   cudaStreamDestroy(c->s_h2d);
+  cudaStreamDestroy(c->s_h2d2);
   c->pinned.destroy();
   delete c;
   g_ctx = nullptr;
@@ -781,7 +1042,7 @@ cswap_status cswap_set_format(const cswap_format* f) {
 }
 
 cswap_status cswap_set_zvc_launch(uint32_t grid, int32_t variant) {
-  if (!zvc_set_launch(grid, variant)) return fail(CSWAP_ERR_INVALID, "variant %d outside -1..3", int(variant));
+  if (!zvc_set_launch(grid, variant)) return fail(CSWAP_ERR_INVALID, "variant %d outside -1..8", int(variant));
   return CSWAP_OK;
 }
 
@@ -841,7 +1102,7 @@ cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uin
   const uint8_t* inb = static_cast<const uint8_t*>(in);
   uint8_t* tmp = nullptr;
   const uint64_t tmp_bytes = n ? decompress_tmp_bytes(codec, n, f, 0, K) : 0;
-  if (tmp_bytes) CU(cudaMallocAsync(&tmp, tmp_bytes, st));
+  if (tmp_bytes) CU(cudaMallocFromPoolAsync(reinterpret_cast<void**>(&tmp), tmp_bytes, c->pool, st));
   c->launches += 2;  // prep, err merge (+ the codec's kernels)
   cswap_status s = run_group(c, st, group_key(kGrpDecompress, codec, dtype), [&](cudaStream_t gs) {
     TRY(cuda_status(launch_prep(inb, in_size, codec, dtype, n, F, param_of(codec, f), L.b->sc, e, true, gs), "prep"));
@@ -964,6 +1225,7 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     return fail(CSWAP_ERR_NOMEM, "pinned alloc failed");
   }
   auto bail = [&](cswap_status s) {
+    finish_out(h, 2, s, "swap-out not issued");
     cswap_handle_free(h);
     return s;
   };
@@ -972,6 +1234,9 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     return bail(fail(CSWAP_ERR_CUDA, "event create failed"));
   int use = codec;
   if (codec == CSWAP_CODEC_AUTO) {
+    // the selector runs on the host, so AUTO waits for the probe's counts:
+    // the one host synchronisation of the swap-out path.  Fixed codecs (or a replayed plan,
+    // NEXT-2) never block the caller.
     cswap_probe_result p;
     cswap_status s = probe_impl(c, d_in, n, dtype, &p, st);
     if (s != CSWAP_OK) return bail(s);
@@ -985,72 +1250,84 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
   h->codec = use;
   const uint64_t F = f.frame_elems;
   const uint32_t K = uint32_t((n + F - 1) / F);
-  cudaEvent_t ready;
-  if (cudaEventCreateWithFlags(&ready, cudaEventDisableTiming) != cudaSuccess)
-    return bail(fail(CSWAP_ERR_CUDA, "event create failed"));
+  const uint64_t ds = al16(64 + 8ull * K);
   if (use == CSWAP_CODEC_NONE) {
-    // raw offload: host writes header + frame table, the copy engine moves the frames
+    // raw offload (vDNN): the host writes header + frame table, the copy engine
+    // moves the tensor's bytes straight into the frames after the caller's stream reaches here
     const uint64_t cap = max_size(n, w, CSWAP_CODEC_NONE, f);
     h->host = c->pinned.alloc(cap);
     if (!h->host) return bail(fail(CSWAP_ERR_NOMEM, "pinned alloc of %llu B failed", (unsigned long long)cap));
-    std::memset(h->host, 0, al16(64 + 8ull * K));
-    const uint64_t tail = al16(64 + 8ull * K) + uint64_t(w) * n;
-    std::memset(h->host + tail, 0, cap - tail);
-    uint64_t total = al16(64 + 8ull * K);
+    h->cap = cap;
+    const uint64_t tail = ds + uint64_t(w) * n;
+    std::memset(h->host + tail, 0, cap - tail);  // frame padding
+    uint64_t total = ds;
     for (uint32_t k = 0; k < K; k++) {
-      const uint64_t fb = al16(uint64_t(w) * std::min<uint64_t>(F, n - uint64_t(k) * F));
-      std::memcpy(h->host + 64 + 8ull * k, &fb, 8);
-      total += fb;
+      total += al16(uint64_t(w) * std::min<uint64_t>(F, n - uint64_t(k) * F));
+      h->ends.push_back(total);
     }
-    std::memcpy(h->host, "CSWP", 4);
-    const uint16_t ver = 1;
-    std::memcpy(h->host + 4, &ver, 2);
-    h->host[6] = 0;
-    h->host[7] = uint8_t(dtype);
-    std::memcpy(h->host + 8, &n, 8);
-    std::memcpy(h->host + 16, &F, 8);
-    std::memcpy(h->host + 24, &K, 4);
-    std::memcpy(h->host + 32, &total, 8);
+    write_host_header(h);
     h->bytes = total;
     if (n) {
-      if (cudaEventRecord(ready, st) != cudaSuccess || cudaStreamWaitEvent(c->s_d2h, ready, 0) != cudaSuccess ||
-          cudaMemcpyAsync(h->host + al16(64 + 8ull * K), d_in, uint64_t(w) * n, cudaMemcpyDeviceToHost, c->s_d2h) !=
-              cudaSuccess) {
-        cudaEventDestroy(ready);
-        return bail(fail(CSWAP_ERR_CUDA, "raw offload failed"));
-      }
+      cudaEvent_t ready;
+      if (cudaEventCreateWithFlags(&ready, cudaEventDisableTiming) != cudaSuccess)
+        return bail(fail(CSWAP_ERR_CUDA, "event create failed"));
+      const bool ok = cudaEventRecord(ready, st) == cudaSuccess && cudaStreamWaitEvent(c->s_d2h, ready, 0) == cudaSuccess &&
+                      cudaMemcpyAsync(h->host + ds, d_in, uint64_t(w) * n, cudaMemcpyDeviceToHost, c->s_d2h) == cudaSuccess;
+      cudaEventDestroy(ready);
+      if (!ok) return bail(fail(CSWAP_ERR_CUDA, "raw offload failed"));
     }
     cudaEventRecord(h->ev_out, c->s_d2h);
-    cudaEventDestroy(ready);
+    finish_out(h, 1, CSWAP_OK, "");
     *out = h;
     return CSWAP_OK;
   }
-  // compressed offload: compress into stream-ordered device staging, read the size, D2H
+  // compressed offload ("compression in parallel before swapping"; Fig. 2): the
+  // codec writes the container into device staging sized for its worst case and publishes each
+  // finished frame; the executor thread copies frames to the pinned host container as they are
+  // published.  Nothing here waits for the device.
   const uint64_t cap = max_size(n, w, use, f);
   uint8_t* staging = nullptr;
-  cswap_status s = CSWAP_OK;
-  if (cudaMallocAsync(&staging, cap, st) != cudaSuccess) {
-    cudaEventDestroy(ready);
+  if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging), cap, c->pool, st) != cudaSuccess)
     return bail(fail(CSWAP_ERR_NOMEM, "device staging of %llu B failed", (unsigned long long)cap));
+  h->host = c->pinned.alloc(cap);
+  h->cap = cap;
+  uint64_t* prog = reinterpret_cast<uint64_t*>(c->pinned.alloc(8ull * std::max<uint32_t>(K, 1)));
+  if (!h->host || !prog) {
+    cudaFreeAsync(staging, st);
+    c->pinned.free(reinterpret_cast<uint8_t*>(prog));
+    return bail(fail(CSWAP_ERR_NOMEM, "pinned alloc of %llu B failed", (unsigned long long)cap));
   }
-  Timer tm(c, st);
-  s = do_compress(c, d_in, n, dtype, use, f, staging, h->size_slot(), st);
-  tm.stop();
-  if (s == CSWAP_OK && cudaEventRecord(ready, st) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "event record");
-  if (s == CSWAP_OK && cudaEventSynchronize(ready) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "compress failed");
-  if (s == CSWAP_OK) {
-    h->bytes = *h->size_slot();
-    tm.commit(use, 0, n * uint64_t(w), h->bytes);
-    h->host = c->pinned.alloc(h->bytes);
-    if (!h->host) s = fail(CSWAP_ERR_NOMEM, "pinned alloc of %llu B failed", (unsigned long long)h->bytes);
+  std::memset(prog, 0, 8ull * std::max<uint32_t>(K, 1));
+  cswap_status s;
+  cudaEvent_t done = nullptr;
+  {
+    Timer tm(c, st);
+    // the container size goes to the timer's pinned slot when timing (read at collection), else
+    // to a device word nobody reads (the executor takes the size from the progress words)
+    uint64_t* osz = tm.stamps ? tm.stamps + 2 : c->dev_sink;
+    // per-frame publication pays only when the D2H link would otherwise wait for this tensor's
+    // compression (nothing queued ahead of it); CSWAP_FRAME_PUBLISH=0/1 forces it off/on
+    bool frame_publish;
+    if (const char* e = getenv("CSWAP_FRAME_PUBLISH")) {
+      frame_publish = e[0] == '1';
+    } else {
+      std::lock_guard<std::mutex> lk(c->qm);
+      frame_publish = c->q.empty() && cudaStreamQuery(c->s_d2h) == cudaSuccess;
+    }
+    s = do_compress(c, d_in, n, dtype, use, f, staging, osz, st, prog, frame_publish);
+    if (s == CSWAP_OK) tm.commit(use, 0, n * uint64_t(w), 0);
   }
-  if (s == CSWAP_OK && (cudaStreamWaitEvent(c->s_d2h, ready, 0) != cudaSuccess ||
-                        cudaMemcpyAsync(h->host, staging, h->bytes, cudaMemcpyDeviceToHost, c->s_d2h) != cudaSuccess))
-    s = fail(CSWAP_ERR_CUDA, "offload copy failed");
-  cudaFreeAsync(staging, s == CSWAP_OK ? c->s_d2h : st);
-  cudaEventRecord(h->ev_out, c->s_d2h);
-  cudaEventDestroy(ready);
-  if (s != CSWAP_OK) return bail(s);
+  if (s == CSWAP_OK && (cudaEventCreateWithFlags(&done, cudaEventDisableTiming) != cudaSuccess ||
+                        cudaEventRecord(done, st) != cudaSuccess))
+    s = fail(CSWAP_ERR_CUDA, "event record failed");
+  if (s != CSWAP_OK) {
+    if (done) cudaEventDestroy(done);
+    cudaFreeAsync(staging, st);
+    cudaStreamSynchronize(st);  // the group may have been partly enqueued: prog is still referenced
+    c->pinned.free(reinterpret_cast<uint8_t*>(prog));
+    return bail(s);
+  }
+  enqueue_out(c, new OutJob{h, staging, prog, K, done});
   *out = h;
   return CSWAP_OK;
 }
@@ -1060,57 +1337,85 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
   Ctx* c = h->ctx;
   const int w = width(h->dtype);
   if (h->n) TRY(check_common(d_out, "d_out"));
+  TRY(wait_out(h));  // the executor has issued the D2H copies: frame ranges known, ev_out recorded
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const cswap_format& f = h->fmt;
   const uint64_t F = f.frame_elems, n = h->n;
   const uint32_t K = uint32_t((n + F - 1) / F);
-  CU(cudaEventSynchronize(h->ev_out));  // the host container (header, frame table) is complete
+  const uint64_t ds = al16(64 + 8ull * K);
   h->in_issued = true;
   *h->err_slot() = 0;
   if (n == 0) return cudaEventRecord(h->ev_in, st) == cudaSuccess ? CSWAP_OK : fail(CSWAP_ERR_CUDA, "record");
-  cudaEvent_t ready;
-  CU(cudaEventCreateWithFlags(&ready, cudaEventDisableTiming));
-  CU(cudaEventRecord(ready, st));
-  CU(cudaStreamWaitEvent(c->s_h2d, ready, 0));
+  if (h->ends.size() != K || h->ends.back() != h->bytes)
+    return fail(CSWAP_ERR_CORRUPT, "frame ranges of the handle are inconsistent");
+  // the H2D copies are ordered after the D2H on the device (no host wait for the swap-out)
+  CU(cudaStreamWaitEvent(c->s_h2d, h->ev_out, 0));
   if (h->codec == CSWAP_CODEC_NONE) {
-    CU(cudaMemcpyAsync(d_out, h->host + al16(64 + 8ull * K), uint64_t(w) * n, cudaMemcpyHostToDevice, c->s_h2d));
-    CU(cudaEventRecord(h->ev_in, c->s_h2d));
-    CU(cudaStreamWaitEvent(st, h->ev_in, 0));
+    cudaEvent_t ready;
+    CU(cudaEventCreateWithFlags(&ready, cudaEventDisableTiming));
+    cswap_status s = CSWAP_OK;
+    if (cudaEventRecord(ready, st) != cudaSuccess || cudaStreamWaitEvent(c->s_h2d, ready, 0) != cudaSuccess ||
+        cudaMemcpyAsync(d_out, h->host + ds, uint64_t(w) * n, cudaMemcpyHostToDevice, c->s_h2d) != cudaSuccess ||
+        cudaEventRecord(h->ev_in, c->s_h2d) != cudaSuccess || cudaStreamWaitEvent(st, h->ev_in, 0) != cudaSuccess)
+      s = fail(CSWAP_ERR_CUDA, "raw prefetch failed");
     cudaEventDestroy(ready);
-    return CSWAP_OK;
+    return s;
   }
-  // pipelined prefetch: groups of frames of ~64 MiB raw; H2D(g+1) overlaps decompress(g)
-  const uint64_t* fb = reinterpret_cast<const uint64_t*>(h->host + 64);
+  CU(cudaStreamWaitEvent(c->s_h2d2, h->ev_out, 0));
+  // pipelined prefetch per frame (R7; the pipelined cost model's K): frame k's H2D overlaps the
+  // decompression of frame k-1.  Staging is allocated on the first copy stream, which the
+  // second copy stream follows; consecutive frames alternate between the two copy streams.
   uint8_t* staging = nullptr;
-  CU(cudaMallocAsync(&staging, h->bytes, c->s_h2d));
-  const uint64_t group_raw = uint64_t(64) << 20;
-  const uint32_t fpg = uint32_t(std::max<uint64_t>(1, group_raw / (F * w)));
+  if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging), h->bytes, c->pool, c->s_h2d) != cudaSuccess)
+    return fail(CSWAP_ERR_NOMEM, "swap-in staging of %llu B failed", (unsigned long long)h->bytes);
   std::vector<cudaEvent_t> evs;
   cswap_status s = CSWAP_OK;
+  cudaEvent_t alloc_ev;
+  CU(cudaEventCreateWithFlags(&alloc_ev, cudaEventDisableTiming));
+  evs.push_back(alloc_ev);
+  if (cudaEventRecord(alloc_ev, c->s_h2d) != cudaSuccess || cudaStreamWaitEvent(c->s_h2d2, alloc_ev, 0) != cudaSuccess)
+    s = fail(CSWAP_ERR_CUDA, "stream order failed");
+  // pipeline steps: runs of whole frames of >= min_group container bytes (one H2D copy + one
+  // decode launch group each; a copy's DMA ramp / tail costs a few us, so the link runs at
+  // 53.4 GB/s with one copy per 8 MiB frame and 54.7 with ~32 MiB copies)
+  const uint64_t min_group = env_bytes("CSWAP_SWAPIN_GROUP_MB", uint64_t(32) << 20);
+  std::vector<uint32_t> gk{0};
+  {
+    uint64_t start = 0;
+    for (uint32_t k = 0; k < K; k++)
+      if (h->ends[k] - start >= min_group || k + 1 == K) {
+        gk.push_back(k + 1);
+        start = h->ends[k];
+      }
+  }
   {
     Lease L(*c, st, decompress_tiles(n, w, f), decompress_aux(n, w, f));
-    s = L.status;
+    if (s == CSWAP_OK) s = L.status;
     uint32_t* e_dev = L.b->sc.err;  // device word; merged into the handle's pinned slot at the end
     uint64_t off = 0;
-    for (uint32_t k0 = 0; k0 < K && s == CSWAP_OK; k0 += fpg) {
-      const uint32_t k1 = std::min(K, k0 + fpg);
-      uint64_t end = al16(64 + 8ull * K);
-      for (uint32_t k = 0; k < k1; k++) end += fb[k];
-      if (k1 == K) end = h->bytes;
+    uint32_t gi = 0;
+    for (; gi + 1 < gk.size() && s == CSWAP_OK; gi++) {
+      const uint32_t k0 = gk[gi], k1 = gk[gi + 1];
+      const uint64_t end = h->ends[k1 - 1];  // trusted: published by the compress kernels
+      if (end <= off || end > h->bytes) {
+        s = fail(CSWAP_ERR_CORRUPT, "frame range out of bounds");
+        break;
+      }
+      cudaStream_t cs = (gi & 1) ? c->s_h2d2 : c->s_h2d;
       cudaEvent_t e;
       if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) {
         s = fail(CSWAP_ERR_CUDA, "event create");
         break;
       }
       evs.push_back(e);
-      if (cudaMemcpyAsync(staging + off, h->host + off, end - off, cudaMemcpyHostToDevice, c->s_h2d) != cudaSuccess ||
-          cudaEventRecord(e, c->s_h2d) != cudaSuccess || cudaStreamWaitEvent(st, e, 0) != cudaSuccess) {
+      if (cudaMemcpyAsync(staging + off, h->host + off, end - off, cudaMemcpyHostToDevice, cs) != cudaSuccess ||
+          cudaEventRecord(e, cs) != cudaSuccess || cudaStreamWaitEvent(st, e, 0) != cudaSuccess) {
         s = fail(CSWAP_ERR_CUDA, "prefetch copy failed");
         break;
       }
       uint8_t* tmp = nullptr;
       const uint64_t tmp_bytes = decompress_tmp_bytes(h->codec, n, f, k0, k1);
-      if (tmp_bytes && cudaMallocAsync(&tmp, tmp_bytes, st) != cudaSuccess) {
+      if (tmp_bytes && cudaMallocFromPoolAsync(reinterpret_cast<void**>(&tmp), tmp_bytes, c->pool, st) != cudaSuccess) {
         s = fail(CSWAP_ERR_NOMEM, "decode scratch");
         break;
       }
@@ -1134,15 +1439,16 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
       off = end;
     }
   }
+  // every staging read is on st (the last decode); frees and the end event follow it there
   cudaFreeAsync(staging, st);
   cudaEventRecord(h->ev_in, st);
   for (auto e : evs) cudaEventDestroy(e);
-  cudaEventDestroy(ready);
   return s;
 }
 
 cswap_status cswap_handle_wait(cswap_handle* h) {
   if (!h) return fail(CSWAP_ERR_INVALID, "handle is NULL");
+  TRY(wait_out(h));
   CU(cudaEventSynchronize(h->ev_out));
   if (h->in_issued) {
     CU(cudaEventSynchronize(h->ev_in));
@@ -1153,22 +1459,28 @@ cswap_status cswap_handle_wait(cswap_handle* h) {
 
 cswap_status cswap_handle_record_out(cswap_handle* h, void* stream) {
   if (!h) return fail(CSWAP_ERR_INVALID, "handle is NULL");
+  TRY(wait_out(h));
   CU(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), h->ev_out, 0));
   return CSWAP_OK;
 }
 
-cswap_status cswap_handle_query(const cswap_handle* h, cswap_codec* codec, uint64_t* container_bytes,
+cswap_status cswap_handle_query(const cswap_handle* hc, cswap_codec* codec, uint64_t* container_bytes,
                                 const void** host_container, cswap_decision* decision) {
-  if (!h) return fail(CSWAP_ERR_INVALID, "handle is NULL");
+  if (!hc) return fail(CSWAP_ERR_INVALID, "handle is NULL");
+  cswap_handle* h = const_cast<cswap_handle*>(hc);  // waiting on the handle's state is not a change
   if (codec) *codec = cswap_codec(h->codec);
-  if (container_bytes) *container_bytes = h->bytes;
-  if (host_container) *host_container = h->host;
   if (decision) *decision = h->dec;
+  if (container_bytes || host_container) {
+    TRY(wait_out(h));
+    if (container_bytes) *container_bytes = h->bytes;
+    if (host_container) *host_container = h->host;
+  }
   return CSWAP_OK;
 }
 
 void cswap_handle_free(cswap_handle* h) {
   if (!h) return;
+  wait_out(h);  // the executor no longer touches h
   if (h->ev_out) cudaEventSynchronize(h->ev_out);
   if (h->ev_in && h->in_issued) cudaEventSynchronize(h->ev_in);
   if (h->ev_out) cudaEventDestroy(h->ev_out);
@@ -1214,6 +1526,7 @@ uint64_t cswap_collect_kernel_timing(cswap_kernel_record* out, uint64_t cap) {
     if (e.stamps) {  // written by the group's stamp kernels, complete once e.b is
       const volatile uint64_t* t = e.stamps;
       e.r.device_ms = (t[0] && t[1] > t[0]) ? double(t[1] - t[0]) * 1e-6 : 0.0;
+      if (!e.r.comp_bytes) e.r.comp_bytes = t[2];  // swap-out compress: container size
       c->pinned.free(reinterpret_cast<uint8_t*>(e.stamps));
     }
     if (out && k < cap) out[k] = e.r;

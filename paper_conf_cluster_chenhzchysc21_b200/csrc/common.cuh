@@ -1,7 +1,7 @@
 // common.cuh — shared device helpers for the CSWAP sm_100a kernels.
 //
-// Container v1 geometry, the epoch-tagged decoupled-lookback protocol used by
-// the single-pass codec kernels, and small PTX wrappers (acquire/release at .gpu scope).
+// Container v1 geometry, the epoch-tagged per-tile status words polled by the
+// persistent ZVC compress, TMA bulk-copy / mbarrier wrappers and small PTX memory-order helpers.
 #pragma once
 #include <cstdint>
 #include <type_traits>
@@ -28,9 +28,9 @@ __host__ __device__ __forceinline__ uint64_t frame_len(uint64_t n, uint64_t F, u
   return (n - s) < F ? (n - s) : F;
 }
 
-// ---- scratch shared by one launch sequence (owned by the runtime, see runtime.cpp) ----
+// ---- scratch shared by one launch sequence (leased per operation by api.cu) ----
 struct Scratch {
-  uint64_t* status;       // per-tile lookback word: value<<16 | epoch<<2 | flag
+  uint64_t* status;       // per-tile status word: value<<16 | epoch<<2 | flag
   uint32_t* tickets;      // per-epoch tile-ticket counters (zeroed slots)
   uint64_t* aux;          // per-frame / per-block u64 scratch (frame starts, block offsets ...)
   uint64_t* aux2;         // second per-frame / per-tile array
@@ -39,7 +39,20 @@ struct Scratch {
   uint64_t* tbuf2;        // second per-tile array, 32 bytes per tile (u64, or CSR: u32[8] slab counts)
   uint64_t* aux3;         // third per-frame u64 array (run / non-zero totals)
   uint64_t cap_tiles, cap_aux;
+  // swap-out progress (NULL outside cswap_swap_out): host-mapped pinned u64[K]; the compress
+  // group stores kProgReady | (end offset of frame k in the container) once every byte of frame
+  // k (and its frame-table entry) is in device memory, so the host can start that frame's D2H
+  uint64_t* prog;
 };
+constexpr uint64_t kProgReady = 1ull << 63;
+
+// Publish "frame k complete, ends at byte `end`" to host-mapped memory.  The caller has made the
+// frame's stores visible at gpu scope (acq_rel chain or a kernel boundary); the copy engine
+// that the host then starts reads device memory through L2, so no system-scope fence is needed
+// (a fence.sys would wait behind the PCIe write queue of the D2H copies already in flight).
+__device__ __forceinline__ void publish_frame(uint64_t* prog, uint32_t k, uint64_t end) {
+  asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(prog + k), "l"(end | kProgReady) : "memory");
+}
 
 // ---- memory-order helpers -------------------------------------------------------------
 __device__ __forceinline__ uint64_t ld_acquire(const uint64_t* p) {
@@ -79,127 +92,6 @@ __device__ __forceinline__ uint64_t warp_sum_u64(uint64_t v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
   return v;
-}
-
-// Decoupled lookback (single-pass chained scan, CUB style) for tile `tile` inside a segment
-// whose first tile is `seg_first` (< tile).  The segment's first tile publishes only P.
-// Called by one full warp; returns the exclusive prefix (sum of A values + the nearest P).
-__device__ __forceinline__ uint64_t lookback(const uint64_t* status, int64_t tile, int64_t seg_first,
-                                             uint32_t epoch) {
-  const int lane = threadIdx.x & 31;
-  uint64_t excl = 0;
-  int64_t pos = tile - 1;
-  while (true) {
-    const int64_t t = pos - lane;
-    uint64_t s = 0;
-    uint32_t f = 0;
-    bool ok;
-    uint32_t backoff = 32;
-    while (true) {
-      if (t >= seg_first) {
-        s = ld_relaxed(status + t);
-        f = status_flag(s, epoch);
-        ok = f != 0;
-      } else {
-        ok = true;  // below the segment: contributes nothing (a P is always found first)
-        f = 0;
-        s = 0;
-      }
-      if (__all_sync(0xffffffffu, ok)) break;
-      __nanosleep(backoff);
-      backoff = backoff < 512 ? backoff * 2 : 512;
-    }
-    const uint32_t pmask = __ballot_sync(0xffffffffu, t >= seg_first && f == kFlagP);
-    if (pmask) {
-      const int pl = __ffs(pmask) - 1;  // nearest P
-      uint64_t v = (lane <= pl && t >= seg_first) ? status_value(s) : 0;
-      excl += warp_sum_u64(v);
-      return excl;
-    }
-    uint64_t v = (t >= seg_first) ? status_value(s) : 0;
-    excl += warp_sum_u64(v);
-    pos -= 32;
-  }
-}
-
-__device__ __forceinline__ uint64_t warp_suffix_sum_u64(uint64_t v) {  // inclusive, lane l: sum over lanes >= l
-  const int lane = threadIdx.x & 31;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint64_t y = __shfl_down_sync(0xffffffffu, v, o);
-    if (lane + o < 32) v += y;
-  }
-  return v;
-}
-
-// Decoupled lookback that also PUBLISHES inclusive prefixes ("P") for the tiles it walks over
-// (up to the last kHist windows before the P it finds).  Tiles later in ticket order then find
-// a P one window back instead of re-walking the same run of aggregates, which keeps the lookback
-// short when hundreds of tiles are in flight.  Publishing is idempotent: any walker computes the
-// same inclusive value for a tile, and only tiles already flagged A are overwritten.
-template <int kHist = 8>
-__device__ __forceinline__ uint64_t lookback_propagate(uint64_t* status, int64_t tile, int64_t seg_first,
-                                                       uint32_t epoch) {
-  const int lane = threadIdx.x & 31;
-  // h[0] = oldest remembered window (closest to `tile`), h[nh-1] = newest; the window in h[k]
-  // covers tiles (pos_P + 32 * (nh - k)) - lane once the P window at pos_P is found.
-  uint64_t h[kHist];
-#pragma unroll
-  for (int k = 0; k < kHist; k++) h[k] = 0;
-  int nh = 0;
-  uint64_t dropped = 0;  // aggregates of windows pushed out of h (closest to `tile`)
-  int64_t pos = tile - 1;
-  while (true) {
-    const int64_t t = pos - lane;
-    const bool inseg = t >= seg_first;
-    uint64_t s = 0;
-    uint32_t f = 0;
-    uint32_t backoff = 32;
-    while (true) {
-      bool ok = true;
-      if (inseg) {
-        s = ld_relaxed(status + t);
-        f = status_flag(s, epoch);
-        ok = f != 0;
-      }
-      if (__all_sync(0xffffffffu, ok)) break;
-      __nanosleep(backoff);
-      backoff = backoff < 512 ? backoff * 2 : 512;
-    }
-    const uint32_t pmask = __ballot_sync(0xffffffffu, inseg && f == kFlagP);
-    if (pmask) {
-      const int pl = __ffs(pmask) - 1;
-      // inclusive value of tile (pos - l), l <= pl: P(pl) + aggregates of lanes l .. pl-1
-      const uint64_t a = lane <= pl ? status_value(s) : 0;
-      const uint64_t incl = warp_suffix_sum_u64(a);
-      if (lane < pl) st_release(status + t, make_status(incl, epoch, kFlagP));
-      uint64_t base = __shfl_sync(0xffffffffu, incl, 0);  // inclusive prefix of tile `pos`
-#pragma unroll
-      for (int k = kHist - 1; k >= 0; k--) {
-        if (k < nh) {
-          const int64_t tp = pos + 32 * (nh - k) - lane;
-          const uint64_t in2 = warp_suffix_sum_u64(h[k]) + base;
-          st_release(status + tp, make_status(in2, epoch, kFlagP));  // these windows are all in-segment
-          base = __shfl_sync(0xffffffffu, in2, 0);
-        }
-      }
-      return base + dropped;
-    }
-    // no P here: remember this window's aggregates (all lanes are in-segment, else a P existed)
-    const uint64_t av = status_value(s);
-    if (nh == kHist) {
-      dropped += warp_sum_u64(h[0]);
-#pragma unroll
-      for (int k = 0; k < kHist - 1; k++) h[k] = h[k + 1];
-      h[kHist - 1] = av;
-    } else {
-#pragma unroll
-      for (int k = 0; k < kHist; k++)
-        if (k == nh) h[k] = av;
-      nh++;
-    }
-    pos -= 32;
-  }
 }
 
 __device__ __forceinline__ void set_error(uint32_t* err, uint32_t code) {

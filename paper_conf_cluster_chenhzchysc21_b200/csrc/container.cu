@@ -311,3 +311,45 @@ cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, c
 }
 
 }  // namespace cswap
+
+namespace cswap {
+// Swap-out progress for the multi-pass codecs (RLE, CSR, LZ4, NONE): launched after the group's
+// last kernel, so every frame is complete; writes kProgReady | end offset of each frame from the
+// container's frame table (one CTA: per-thread chunk sums, block scan, per-thread writes).
+__global__ void __launch_bounds__(1024) publish_frames_kernel(const uint8_t* out, uint32_t K, uint64_t* prog) {
+  __shared__ uint64_t s_w[33];
+  const uint64_t* fb = reinterpret_cast<const uint64_t*>(out + 64);
+  const uint32_t per = (K + blockDim.x - 1) / blockDim.x, k0 = threadIdx.x * per, k1 = umin32(K, k0 + per);
+  uint64_t sum = 0;
+  for (uint32_t k = k0; k < k1; k++) sum += fb[k];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t inc = sum;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint64_t y = __shfl_up_sync(0xffffffffu, inc, o);
+    if (lane >= o) inc += y;
+  }
+  if (lane == 31) s_w[warp] = inc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint64_t acc = 0;
+    for (int w = 0; w < int(blockDim.x / 32); w++) {
+      const uint64_t x = s_w[w];
+      s_w[w] = acc;
+      acc += x;
+    }
+  }
+  __syncthreads();
+  uint64_t end = data_start(K) + s_w[warp] + inc - sum;
+  for (uint32_t k = k0; k < k1; k++) {
+    end += fb[k];
+    publish_frame(prog, k, end);
+  }
+}
+
+cudaError_t launch_publish_frames(const uint8_t* out, uint32_t K, uint64_t* prog, cudaStream_t st) {
+  if (!K) return cudaSuccess;
+  publish_frames_kernel<<<1, 1024, 0, st>>>(out, K, prog);
+  return cudaGetLastError();
+}
+}  // namespace cswap

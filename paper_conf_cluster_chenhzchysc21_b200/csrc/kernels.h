@@ -30,6 +30,8 @@ cudaError_t launch_none_decompress(const uint8_t* in, void* out, uint64_t n, int
                                    uint32_t* err, cudaStream_t st);
 cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, const Scratch& sc, uint32_t epoch,
                          cudaStream_t st);
+// swap-out progress of a finished compress group: prog[k] = kProgReady | end offset of frame k
+cudaError_t launch_publish_frames(const uint8_t* out, uint32_t K, uint64_t* prog, cudaStream_t st);
 
 // zvc.cu
 uint32_t zvc_tiles(uint64_t n, int w, uint64_t F, uint32_t k0, uint32_t k1, uint32_t* tpf_out);

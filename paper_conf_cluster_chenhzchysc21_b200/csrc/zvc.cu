@@ -5,13 +5,13 @@
 // Byte layout: DESIGN.md §3 (frame = u32 bitmap[ceil(Fk/32)] pad16 | non-zero words pad16).
 //
 // Compress (one pass over the input): a persistent, warp-specialised kernel.
-//   warp 8  (producer): claims 32 KiB tiles in ticket order and streams them into a ring of
-//           shared-memory stages with cp.async.bulk (TMA 1-D) + mbarrier completion;
-//   warps 0-7 (consumers): count tile i+1 (warp ballots -> bitmap words, per-lane ranks) while
-//           the scan warp resolves tile i, then compact tile i at its container offset and store
-//           it with 128-bit stores;
-//   warp 9  (scan): publishes each tile's byte count and resolves its absolute container
-//           offset by decoupled lookback (frame k's first tile chains on frame k-1's end).
+//   producer warp: streams the CTA's tiles (static round robin) into a ring of shared-memory
+//           stages with cp.async.bulk (TMA 1-D) + mbarrier completion;
+//   consumer warps: count tile i (warp ballots -> bitmap words, per-lane ranks, in-place
+//           compaction) and publish its count, then emit tile i-LAG at its container offset;
+//   resolver warps (one per stage): the tile's absolute offset from the published COUNTS of the
+//           earlier tiles of its frame (per-frame and 32-tile-group accumulators), no chained
+//           prefixes.
 // Decompress (no inter-CTA waiting): tile popcounts of the bitmap (reads n/8 B),
 // a per-frame scan of those counts into value offsets, then one CTA per tile pulls its bitmap
 // slice and value span into shared memory with cp.async.bulk and expands with 128-bit stores.
@@ -209,10 +209,39 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
   };
 
   if (warp == kProducerWarp) {  // ----------------------------------------- producer (TMA)
-    for (uint32_t i = 0;; i++) {
+    // swap-out progress (sc.prog): once a stage's previous tile is fully emitted (bar_empty:
+    // every consumer warp arrived after its stores, mbarrier arrive = release.cta, wait =
+    // acquire.cta), count it for its frame with a gpu-scope acq_rel atomic; the CTA that
+    // completes a frame publishes the frame's end offset (frame start + its frame-table entry,
+    // both written before the frame's last tiles were emitted) for the host's per-frame D2H
+    uint64_t* const fdone = sc.aux2 + K + uint64_t(K) * gpf;  // zeroed with the accumulators
+    auto tile_emitted = [&](uint32_t t) {
+      if (!sc.prog || lane != 0) return;
+      uint32_t k, j, te, be;
+      uint64_t Fk;
+      tile_geom(t, k, j, Fk, te, be);
+      unsigned long long old;
+      asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;"
+                   : "=l"(old)
+                   : "l"(fdone + k)
+                   : "memory");
+      if (old + 1 == cdiv(Fk, G::TILE)) {
+        const uint64_t fs = status_value(ld_relaxed(sc.aux + k));
+        const uint64_t fb = ld_relaxed(reinterpret_cast<const uint64_t*>(out + 64) + k);
+        publish_frame(sc.prog, k, fs + fb);
+      }
+    };
+    uint32_t i = 0;
+    for (;; i++) {
       const int s = i % S;
       long long c0 = clock64();
-      if (i >= S) mbar_wait_sleep(&bar_empty[s], ((i / S) - 1) & 1, kProducerSleep);
+      // the tile of round i - S (this stage's previous tile); counted for its frame only after
+      // the stage is refilled, so the atomic's round trip never delays the next TMA load
+      uint32_t done_t = SENT;
+      if (i >= S) {
+        mbar_wait_sleep(&bar_empty[s], ((i / S) - 1) & 1, kProducerSleep);
+        done_t = s_ticket[s];
+      }
       if (lane == 0) ZPROF_ADD(0, clock64() - c0);
       // static round-robin assignment: CTA b takes tiles b, b + G, b + 2G, ... so every CTA
       // counts the tiles of round r at about the same time and a tile's offset waits only for
@@ -224,6 +253,14 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         if (lane == 0) {
           s_ticket[s] = SENT;
           mbar_arrive(&bar_full[s]);
+        }
+        if (done_t != SENT) tile_emitted(done_t);
+        // the tiles of rounds i-S+1 .. i-1 are still being emitted: wait for each and count it
+        if (sc.prog) {
+          for (uint32_t p = i >= uint32_t(S - 1) ? i - (S - 1) : 0; p < i; p++) {
+            mbar_wait_sleep(&bar_empty[p % S], (p / S) & 1, kProducerSleep);
+            tile_emitted(s_ticket[p % S]);
+          }
         }
         break;
       }
@@ -239,6 +276,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           mbar_arrive(&bar_full[s]);
         }
       }
+      if (done_t != SENT) tile_emitted(done_t);
     }
     return;
   }
@@ -809,6 +847,17 @@ static int prof_enabled() {
   return p;
 }
 
+// CSWAP_ZVC_COOP=0 launches the persistent compress non-cooperatively (A/B measurements only:
+// without it the kernel can stall behind concurrent kernels)
+static bool coop_enabled() {
+  static int c = -1;
+  if (c < 0) {
+    const char* e = getenv("CSWAP_ZVC_COOP");
+    c = (e && e[0] == '0') ? 0 : 1;
+  }
+  return c == 1;
+}
+
 static int sm_count() {
   static int sms = 0;
   if (!sms) {
@@ -827,20 +876,38 @@ static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uin
   const uint32_t TILE = TB / sizeof(T);
   const uint32_t tpf = uint32_t(cdiv(F, TILE));
   const uint32_t tiles = (K - 1) * tpf + uint32_t(cdiv(frame_len(n, F, K - 1), TILE));
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(zvc_compress_persistent<T, S, CW, TB>, cudaFuncAttributeMaxDynamicSharedMemorySize, L::bytes);
-    attr = true;
+  auto kern = zvc_compress_persistent<T, S, CW, TB>;
+  constexpr int threads = compress_threads<S, CW>();
+  static int per_sm = 0;  // resident CTAs per SM, from the occupancy calculator (not the estimate)
+  if (!per_sm) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, L::bytes);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, L::bytes) != cudaSuccess || per_sm < 1)
+      return cudaErrorInvalidConfiguration;
   }
-  const uint32_t per_sm = L::ctas_per_sm;
   // per-frame and per-group (tiles, nnz) accumulators
-  launch_zero_words(sc.aux2, (uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32)) * 2, st);
-  const uint32_t cap = uint32_t(sm_count()) * per_sm;  // co-resident maximum (forward progress)
+  // (+ K per-frame emitted-tile counters for the swap-out progress words)
+  launch_zero_words(sc.aux2, (2 * uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32)) * 2, st);
+  const uint32_t cap = uint32_t(sm_count()) * uint32_t(per_sm);  // co-resident maximum
   const uint32_t want = g_zvc_grid.load(std::memory_order_relaxed);
   const uint32_t grid = std::min<uint32_t>(tiles, want ? std::min(want, cap) : cap);
   timing_kernel_start(st);
-  zvc_compress_persistent<T, S, CW, TB><<<grid, compress_threads<S, CW>(), L::bytes, st>>>(
-      static_cast<const T*>(in), n, F, K, tpf, tiles, out, out_size, sc, epoch, dtype, prof_enabled());
+  // Forward progress: a tile waits for the COUNTS of earlier tiles, which other CTAs produce, so
+  // every CTA of the grid must be resident at once.  A cooperative launch guarantees that (the
+  // grid is admitted only when all of it fits), also while other kernels occupy part of the GPU
+  // or a second compress runs on another stream (tests/test_gpu_concurrency.py).
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(threads);
+  cfg.dynamicSmemBytes = L::bytes;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = coop_enabled() ? 1 : 0;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  const cudaError_t e = cudaLaunchKernelEx(&cfg, kern, static_cast<const T*>(in), n, F, K, tpf, tiles, out, out_size,
+                                           sc, epoch, dtype, prof_enabled());
+  if (e != cudaSuccess) return e;
   if (prof_enabled()) {
     unsigned long long h[16];
     cudaStreamSynchronize(st);
@@ -903,7 +970,7 @@ static cudaError_t launch_compress_t(const void* in, uint64_t n, uint64_t F, uin
 void zvc_compress_scratch(uint64_t n, int w, uint64_t F, uint64_t* tiles, uint64_t* aux) {
   const uint64_t TILE = 16384 / w, K = cdiv(n, F), tpf = cdiv(F, TILE);
   *tiles = K ? (K - 1) * tpf + cdiv(frame_len(n, F, K - 1), TILE) : 0;
-  *aux = K + K * ((tpf + 31) / 32) + 2;
+  *aux = 2 * K + K * ((tpf + 31) / 32) + 2;
 }
 
 cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,

@@ -241,7 +241,15 @@ class Handle:
     def record_out(self, stream=None):
         _check(_L.cswap_handle_record_out(self.raw, _stream(stream)), "cswap_handle_record_out")
 
+    def codec(self) -> int:
+        """The codec the swap-out used (known when cswap_swap_out returns; does not wait)."""
+        c = ctypes.c_int()
+        _check(_L.cswap_handle_query(self.raw, ctypes.byref(c), None, None, None), "cswap_handle_query")
+        return c.value
+
     def query(self):
+        """Codec, container bytes, host pointer and decision; waits until the swap-out's copies
+        are issued (not for the device)."""
         codec = ctypes.c_int()
         nbytes = ctypes.c_uint64()
         host = ctypes.c_void_p()

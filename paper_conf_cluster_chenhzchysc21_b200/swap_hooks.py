@@ -51,9 +51,12 @@ class CSwapBackend:
         flat = t.reshape(-1)
         h = C.swap_out(flat, flat.numel(), _DTYPES[t.dtype], codec, hidden_f, hidden_b)
         # a raw (NONE) offload reads t on the library's copy stream: t's memory must not be
-        # reused before that copy ends -> order a torch stream after it and tie t to it
-        h.record_out(self.keep)
-        t.record_stream(self.keep)
+        # reused before that copy ends -> order a torch stream after it and tie t to it.  A
+        # compressed swap-out reads t only on the current stream (the codec kernels), so torch's
+        # stream-ordered allocator already keeps t alive long enough, and nothing here waits.
+        if h.codec() == C.NONE:
+            h.record_out(self.keep)
+            t.record_stream(self.keep)
         return h
 
     def swap_in(self, h, out: torch.Tensor, stream: torch.cuda.Stream):

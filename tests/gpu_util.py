@@ -32,6 +32,22 @@ def empty_like_words(n, dtype):
     return torch.empty(max(n, 1), dtype=torch.int32 if dtype == 0 else torch.int16, device="cuda")
 
 
+def poisoned_words(n, dtype):
+    """Output buffer filled with 0xA5 bytes: a decoder that skips writing any element (zeros
+    included) leaves the poison there, whatever the allocator happened to return."""
+    t = empty_like_words(n, dtype)
+    t.fill_(-0x5A5A5A5B if dtype == 0 else -0x5A5B)  # 0xA5A5A5A5 / 0xA5A5
+    return t
+
+
+def poison_like(t):
+    """0xA5-filled tensor with t's shape / dtype / device."""
+    import torch
+    out = torch.empty_like(t)
+    out.view(torch.uint8).fill_(0xA5)
+    return out
+
+
 def gpu_compress(C, x: np.ndarray, codec: int, dtype: int, fmt=None, stream=None) -> bytes:
     import torch
     n = x.size
@@ -48,7 +64,7 @@ def gpu_decompress(C, blob: bytes, n: int, dtype: int, codec: int, fmt=None):
     """Returns (words, err)."""
     import torch
     src = torch.from_numpy(np.frombuffer(blob, dtype=np.uint8).copy()).cuda()
-    out = empty_like_words(n, dtype)
+    out = poisoned_words(n, dtype)
     err = torch.zeros(1, dtype=torch.int32, device="cuda")
     C.decompress(src, len(blob), out, n, dtype, codec, fmt=fmt, err=err)
     torch.cuda.synchronize()

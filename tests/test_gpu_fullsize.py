@@ -55,7 +55,7 @@ def test_full_size_sampled_frames(C, codec, dtype, n):
     for k in sorted({0, 1, K // 2, K - 1}):
         ref = O.compress(x[k * F:(k + 1) * F], codec, dtype, F=F, param=prm)
         assert blob[starts[k]:starts[k] + fb[k]] == ref[ds:], f"frame {k}"
-    out = torch.empty_like(d)
+    out = G.poison_like(d)
     h.swap_in(out)
     h.wait()
     assert torch.equal(out, d)

@@ -29,7 +29,7 @@ def test_swap_uses_graphs(C):
     d = G.to_dev(x)
     g0, _ = C.graph_stats()
     h = C.swap_out(d, n, C.F32, C.ZVC)
-    out = G.empty_like_words(n, 0)
+    out = G.poisoned_words(n, 0)
     h.swap_in(out)
     h.wait()
     torch.cuda.synchronize()
@@ -58,7 +58,7 @@ def test_graph_reuse_across_sizes(C, codec):
                 h = C.swap_out(d, n, dt, codec)
                 h.wait()
                 assert h.host_bytes() == ref
-                out = G.empty_like_words(n, dt)
+                out = G.poisoned_words(n, dt)
                 h.swap_in(out)
                 h.wait()
                 torch.cuda.synchronize()
@@ -81,7 +81,7 @@ def test_plain_launch_path_matches():
         "    d = G.to_dev(x)\n"
         "    h = C.swap_out(d, n, 0, codec); h.wait()\n"
         "    assert h.host_bytes() == O.compress(x, codec, 0), codec\n"
-        "    out = G.empty_like_words(n, 0); h.swap_in(out); h.wait(); torch.cuda.synchronize()\n"
+        "    out = G.poisoned_words(n, 0); h.swap_in(out); h.wait(); torch.cuda.synchronize()\n"
         "    assert np.array_equal(G.from_dev(out)[:n], x), codec\n"
         "    h.close()\n"
         "assert C.graph_stats()[0] == 0\n"
@@ -116,7 +116,7 @@ def test_timing_records_carry_device_clock(C):
     n = 8 << 20
     x = synth.relu_iid(n, 0.5, seed=5)
     d = G.to_dev(x)
-    out = G.empty_like_words(n, 0)
+    out = G.poisoned_words(n, 0)
     C.collect_kernel_timing()
     C.set_kernel_timing(True)
     try:

@@ -27,8 +27,7 @@ def test_swap_container_equals_oracle(C, codec, n):
     h.wait()
     ref = O.compress(x, codec, O.F32, F=1 << 20, param={3: 1024, 4: 65536}.get(codec, 0))
     assert h.host_bytes() == ref
-    out = G.empty_like_words(n, 0)
-    out.fill_(-1)
+    out = G.poisoned_words(n, 0)
     h.swap_in(out)
     h.wait()
     torch.cuda.synchronize()
@@ -92,7 +91,7 @@ def test_vgg_sized_tensor_roundtrip_sampled_frames(C):
         Fk = min(F, n - k * F)
         nnz_k = int(torch.count_nonzero(d[k * F:k * F + Fk]).item())
         assert fb[k] == ((Fk + 31) // 32 * 4 + 15) // 16 * 16 + (4 * nnz_k + 15) // 16 * 16
-    out = torch.empty_like(d)
+    out = G.poison_like(d)
     h.swap_in(out)
     h.wait()
     assert torch.equal(out, d)

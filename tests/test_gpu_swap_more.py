@@ -32,7 +32,7 @@ def test_swap_16bit_container_equals_oracle(C, dtype, codec):
     h = C.swap_out(d, n, dtype, codec)
     h.wait()
     assert h.host_bytes() == O.compress(x, codec, dtype, F=1 << 20, param={3: 1024, 4: 65536}.get(codec, 0))
-    out = G.empty_like_words(n, dtype)
+    out = G.poisoned_words(n, dtype)
     h.swap_in(out)
     h.wait()
     torch.cuda.synchronize()
@@ -54,7 +54,7 @@ def test_forward_out_reverse_in_schedule_mixed_codecs(C):
         hs.append(C.swap_out(G.to_dev(x), n, C.F32, codec))
     outs = []
     for x, h in reversed(list(zip(xs, hs))):
-        o = G.empty_like_words(x.size, 0)
+        o = G.poisoned_words(x.size, 0)
         h.swap_in(o)
         outs.append(o)
     outs.reverse()
@@ -79,7 +79,7 @@ def test_swap_on_side_stream_orders_after_pending_work(C):
         torch.cuda._sleep(2_000_000)  # keep the stream busy, then fill d
         d.copy_(src)
         h = C.swap_out(d, n, C.F32, C.ZVC, stream=s)
-        out = torch.empty_like(d)
+        out = G.poison_like(d)
         h.swap_in(out, stream=s)
     s.synchronize()
     h.wait()
@@ -99,7 +99,7 @@ def test_corrupted_host_container_reported_by_wait(C, codec):
     # flip the first frame-table entry (bytes 64..71): frame sizes no longer add up
     p = ctypes.cast(q["host"] + 64, ctypes.POINTER(ctypes.c_uint8))
     p[0] ^= 0x10
-    out = G.empty_like_words(n, 0)
+    out = G.poisoned_words(n, 0)
     h.swap_in(out)
     with pytest.raises(C.CswapError) as e:
         h.wait()
@@ -115,7 +115,7 @@ def test_library_error_word(C):
     blob = bytearray(O.compress(x, O.ZVC, O.F32, F=1024))
     blob[0] ^= 1
     src = torch.from_numpy(np.frombuffer(bytes(blob), np.uint8).copy()).cuda()
-    out = G.empty_like_words(n, 0)
+    out = G.poisoned_words(n, 0)
     C.decompress(src, len(blob), out, n, C.F32, C.ZVC, fmt=(1024, 1024, 65536))  # err = NULL
     with pytest.raises(C.CswapError) as e:
         C.check_device_error()
@@ -145,7 +145,7 @@ def test_bert_like_fp16_set_selection(C):
         assert q["codec"] == ref["codec"], name
         if s == 0.0:
             assert q["codec"] == O.NONE, name
-        out = G.empty_like_words(n, O.F16)
+        out = G.poisoned_words(n, O.F16)
         h.swap_in(out)
         h.wait()
         torch.cuda.synchronize()
