@@ -73,7 +73,9 @@ typedef struct {
  * beta[codec-1][dir][band][i]: t = b0 + b1*S + b2*S*s, dir 0 = compress, 1 = decompress,
  * bands [0,.2) [.2,.35) [.35,.5) [.5,.65) [.65,.8) [.8,1] of the probed sparsity s, S = raw bytes.
  * LZ4 size model: w*nnz + gamma1*zero_runs + gamma2*w*zeros/255.
- * mode 0 = pipelined (frames overlap codec and copy; margin m), 1 = paper (Eq. 2, m = 0). */
+ * mode 0 = pipelined (frames overlap codec and copy; margin m), 1 = paper (Eq. 2, m = 0).
+ * group_bytes: container bytes per swap-in pipeline step (H2D + decode of whole frames); the
+ * pipelined model's swap-in depth G = ceil(K / ceil(group_bytes / frame bytes)), 0 = per frame. */
 typedef struct {
   double alpha_d2h, bw_d2h, alpha_h2d, bw_h2d;
   double beta[4][2][6][3];
@@ -83,6 +85,7 @@ typedef struct {
   int32_t reserved;
   uint64_t frame_elems; /* F used to predict sizes and pipeline depth */
   uint32_t csr_row, lz4_block;
+  double group_bytes;   /* swap-in pipeline step (default 32 MiB) */
 } cswap_calib;
 
 /* Output of the selector: codec (CSWAP_CODEC_NONE or 1..4), predicted T(c*) and T' (s),

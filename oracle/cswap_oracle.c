@@ -21,6 +21,7 @@
 #include <stdint.h>
 #include <stddef.h>
 #include <string.h>
+#include <math.h>
 #include <stdlib.h>
 
 #define ORC_OK 0
@@ -512,6 +513,7 @@ typedef struct {
     int32_t pad_;
     uint64_t frame_elems;                           /* F */
     uint32_t csr_row, lz4_block;                    /* C, B */
+    double group_bytes;                             /* swap-in pipeline step (R22) */
 } orc_calib;
 
 static int band_of(double s) {
@@ -588,8 +590,25 @@ int orc_select(uint64_t n, int dtype, const uint64_t counts[5], double hidden_f,
             /* Eq. 2: T = Time_c + Time_dc + O_f + O_b */
             T = tc + tdc + dmax(xo - hidden_f, 0.0) + dmax(xi - hidden_b, 0.0);
         } else {
-            double Tout = dmax(tc, xo) + dmin(tc, xo) / (double)K;
-            double Tin = dmax(tdc, xi) + dmin(tdc, xi) / (double)K;
+            /* pipelined mode models the executor it predicts (R11, R22).
+             * Swap-out: ZVC hands every finished frame to the copy engine while later frames
+             * are compressed -> a K-step pipeline; RLE, CSR and LZ4 place a frame only after
+             * every frame has been counted / parsed -> codec time then transfer. */
+            double Tout;
+            if (c == C_ZVC)
+                Tout = dmax(tc, xo) + dmin(tc, xo) / (double)K;
+            else
+                Tout = tc + xo;
+            /* Swap-in: H2D + decode in groups of whole frames of >= group_bytes container
+             * bytes: G = ceil(K / q), q = ceil(group_bytes / frame bytes), frames of equal
+             * size (size - header) / K; group_bytes <= 0 -> one frame per step (G = K). */
+            double G = (double)K;
+            double sf = (size - (double)data_start((uint32_t)K)) / (double)K;
+            if (cal->group_bytes > 0 && sf > 0) {
+                double q = ceil(cal->group_bytes / sf);
+                G = ceil((double)K / q);
+            }
+            double Tin = dmax(tdc, xi) + dmin(tdc, xi) / G;
             T = dmax(Tout - hidden_f, 0.0) + dmax(Tin - hidden_b, 0.0);
         }
         out[3 + c - 1] = T;

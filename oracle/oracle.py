@@ -29,7 +29,7 @@ def build(force: bool = False) -> str:
     """Compile the oracle with plain gcc -O2 (scalar C, no SIMD intrinsics)."""
     if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-Wall", "-Wextra", "-fPIC", "-shared",
-                               "-o", LIB, SRC])
+                               "-o", LIB, SRC, "-lm"])
     return LIB
 
 
@@ -43,6 +43,7 @@ class Calib(ctypes.Structure):
         ("mode", ctypes.c_int32), ("pad_", ctypes.c_int32),
         ("frame_elems", ctypes.c_uint64),
         ("csr_row", ctypes.c_uint32), ("lz4_block", ctypes.c_uint32),
+        ("group_bytes", ctypes.c_double),
     ]
 
 
@@ -160,7 +161,7 @@ def probe_estimates(n: int, counts) -> tuple:
 
 def make_calib(alpha_d2h=0.0, bw_d2h=50e9, alpha_h2d=0.0, bw_h2d=50e9, beta=None, lz4_gamma1=3.0,
                lz4_gamma2=1.0, margin=0.05, mode=0, frame_elems=DEFAULT_F, csr_row=DEFAULT_C,
-               lz4_block=DEFAULT_B) -> Calib:
+               lz4_block=DEFAULT_B, group_bytes=float(32 << 20)) -> Calib:
     """beta: array-like [4 codecs][2 dirs][6 bands][3] (defaults to zeros)."""
     c = Calib()
     c.alpha_d2h, c.bw_d2h, c.alpha_h2d, c.bw_h2d = alpha_d2h, bw_d2h, alpha_h2d, bw_h2d
@@ -169,6 +170,7 @@ def make_calib(alpha_d2h=0.0, bw_d2h=50e9, alpha_h2d=0.0, bw_h2d=50e9, beta=None
         c.beta[i] = float(v)
     c.lz4_gamma1, c.lz4_gamma2, c.margin, c.mode = lz4_gamma1, lz4_gamma2, margin, mode
     c.frame_elems, c.csr_row, c.lz4_block = frame_elems, csr_row, lz4_block
+    c.group_bytes = group_bytes
     return c
 
 

@@ -166,6 +166,8 @@ def calib_from_json(d: dict):
                 cal.beta[i] = v
         elif f in d:
             setattr(cal, f, d[f])
+    if "group_bytes" not in d:  # calibrations written before the swap-in group size existed
+        cal.group_bytes = float(32 << 20)
     return cal
 
 

@@ -91,9 +91,19 @@ void decide(uint64_t n, int w, const cswap_probe_result& p, double hf, double hb
     if (paper) {
       T = tc + tdc + std::fmax(xo - hf, 0.0) + std::fmax(xi - hb, 0.0);  // Eq. 2
     } else {
+      // the pipeline the runtime executes (R11, R22): ZVC publishes frames from its
+      // persistent kernel (K-step swap-out pipeline); RLE / CSR / LZ4 place frames only after
+      // counting / parsing every frame (codec time, then transfer); swap-in runs H2D + decode in
+      // groups of whole frames of >= group_bytes container bytes
       const double Kd = double(K);
-      const double Tout = std::fmax(tc, xo) + std::fmin(tc, xo) / Kd;
-      const double Tin = std::fmax(tdc, xi) + std::fmin(tdc, xi) / Kd;
+      const double Tout = ci == 0 ? std::fmax(tc, xo) + std::fmin(tc, xo) / Kd : tc + xo;
+      double G = Kd;
+      const double sf = (size - double(hdr)) / Kd;
+      if (c.group_bytes > 0 && sf > 0) {
+        const double q = std::ceil(c.group_bytes / sf);
+        G = std::ceil(Kd / q);
+      }
+      const double Tin = std::fmax(tdc, xi) + std::fmin(tdc, xi) / G;
       T = std::fmax(Tout - hf, 0.0) + std::fmax(Tin - hb, 0.0);
     }
     out->t_codec[ci] = T;
@@ -207,6 +217,7 @@ void default_calib(cswap_calib* c) {
   c->frame_elems = uint64_t(1) << 22;
   c->csr_row = 1024;
   c->lz4_block = 65536;
+  c->group_bytes = double(uint64_t(32) << 20);
 }
 
 }  // namespace cswap

@@ -56,6 +56,7 @@ class Calib(ctypes.Structure):
         ("mode", ctypes.c_int32), ("reserved", ctypes.c_int32),
         ("frame_elems", ctypes.c_uint64),
         ("csr_row", ctypes.c_uint32), ("lz4_block", ctypes.c_uint32),
+        ("group_bytes", ctypes.c_double),
     ]
 
 

@@ -140,8 +140,9 @@ def test_pipelined_overlap_formula():
     """K frames overlap codec and copy: T_out = max(tc, x) + min(tc, x)/K."""
     n = 1 << 22
     F = 1 << 20
+    # group_bytes = 0: one frame per swap-in step, so both directions are K-step pipelines
     cal = O.make_calib(bw_d2h=50e9, bw_h2d=50e9, beta=beta_const(1e-3, 2e-3), frame_elems=F, mode=0,
-                       margin=0.0)
+                       margin=0.0, group_bytes=0.0)
     x = synth.relu_iid(1 << 18, 0.5, seed=1, exact=True)
     counts = O.probe(x, O.F32)
     r = O.select(n, O.F32, counts, 0, 0, cal)

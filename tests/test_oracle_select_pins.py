@@ -152,20 +152,42 @@ def test_alpha_enters_t_prime_and_t_pipelined_single_frame():
     assert r["codec"] == CSR and r["t_pred"] == r["t_codec"][CSR - 1]
 
 
-def test_alpha_with_four_frames():
+@pytest.mark.parametrize("group_bytes,t_zvc", [
+    (0.0, 1.4e-5),            # one frame per swap-in step: G = K = 4, T_in = 8e-6 + 3e-6/4
+    (256.0, 1.475e-5),        # frames of (608 - 96)/4 = 128 B, q = 2 per step: G = 2, T_in = 8e-6 + 3e-6/2
+    (float(32 << 20), 1.625e-5),  # one step: G = 1, T_in = 8e-6 + 3e-6
+])
+def test_alpha_with_four_frames_and_swap_in_groups(group_bytes, t_zvc):
     b = np.zeros((4, 2, 6, 3))
     b[:, 0, 5, 0] = 1e-6
     b[:, 1, 5, 0] = 8e-6
     cal = O.make_calib(alpha_d2h=4e-6, bw_d2h=6.08e8, alpha_h2d=1e-6, bw_h2d=3.04e8, beta=b, mode=0,
-                       frame_elems=1024)
+                       frame_elems=1024, group_bytes=group_bytes)
     r = O.select(4096, O.F32, (4096, 1, 0, 4096, 4095), 0.0, 0.0, cal)
     # K = 4; ZVC size = align16(64 + 32) + 4 * align16(128) + 0 = 96 + 512 = 608
-    # x_o = 4e-6 + 608/6.08e8 = 5e-6; T_out = max(1e-6, 5e-6) + min/4 = 5.25e-6
-    # x_i = 1e-6 + 608/3.04e8 = 3e-6;  T_in = 8e-6 + 3e-6/4 = 8.75e-6
+    # x_o = 4e-6 + 608/6.08e8 = 5e-6; ZVC swap-out is a K-step pipeline: T_out = 5e-6 + 1e-6/4 = 5.25e-6
+    # x_i = 1e-6 + 608/3.04e8 = 3e-6; T_in = 8e-6 + 3e-6/G
     assert r["size"][ZVC - 1] == 608
-    assert r["t_codec"][ZVC - 1] == pytest.approx(1.4e-5, rel=1e-9)
+    assert r["t_codec"][ZVC - 1] == pytest.approx(t_zvc, rel=1e-9)
     # T' = (4e-6 + 16384/6.08e8) + (1e-6 + 16384/3.04e8)
     assert r["t_prime"] == pytest.approx(5e-6 + 16384 / 6.08e8 + 16384 / 3.04e8, rel=1e-12)
+
+
+def test_multi_pass_codecs_swap_out_is_codec_time_then_transfer():
+    """RLE / CSR / LZ4 place a frame only after every frame is counted / parsed (R22),
+    so their pipelined T_out is t_c + x_o, not the K-step overlap ZVC gets."""
+    b = np.zeros((4, 2, 6, 3))
+    b[:, 0, 5, 0] = 2e-6
+    b[:, 1, 5, 0] = 1e-6
+    cal = O.make_calib(alpha_d2h=4e-6, bw_d2h=6.08e8, alpha_h2d=1e-6, bw_h2d=3.04e8, beta=b, mode=0,
+                       frame_elems=1024)
+    r = O.select(4096, O.F32, (4096, 1, 0, 4096, 4095), 0.0, 0.0, cal)
+    # RLE: r = 1 + (K - 1) = 4 runs: 96 + 4 x 16 + align16(16) + align16(16) = 192 B
+    assert r["size"][RLE - 1] == 192
+    # T_out = 2e-6 + (4e-6 + 192/6.08e8); T_in (one step) = max(1e-6, x_i) + min(...) = 1e-6 + 1e-6 + 192/3.04e8
+    assert r["t_codec"][RLE - 1] == pytest.approx(8e-6 + 192 / 6.08e8 + 192 / 3.04e8, rel=1e-12)
+    # ZVC with the same times overlaps its 4 frames: T_out = max(2e-6, 5e-6) + 2e-6/4 = 5.5e-6
+    assert r["t_codec"][ZVC - 1] == pytest.approx(5.5e-6 + 1e-6 + 3e-6, rel=1e-12)
 
 
 # ------------------------------------------------------------------ paper mode, Eq. 2 with codec times
