@@ -414,6 +414,7 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
     cudaFree(b.sc.tbuf);
     cudaFree(b.sc.tbuf2);
     cudaFree(b.sc.aux3);
+    cudaFree(b.sc.zacc);
   }
   tiles = std::max(tiles, b.sc.cap_tiles * 2);
   aux = std::max(aux, b.sc.cap_aux * 2);
@@ -425,6 +426,7 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
   CU(cudaMalloc(&b.sc.tbuf, tiles * 8));
   CU(cudaMalloc(&b.sc.tbuf2, tiles * 32));  // 32 B per tile: CSR keeps 8 u32 slab counts
   CU(cudaMalloc(&b.sc.aux3, aux * 8));
+  CU(cudaMalloc(&b.sc.zacc, aux * 8));
   CU(cudaMemset(b.sc.status, 0, tiles * 8));
   // epoch-tagged words are also polled in aux (frame starts): a fresh block restarts at epoch 0,
   // so memory recycled from an earlier block could hold words tagged with a live epoch; zero
@@ -432,6 +434,7 @@ cswap_status ensure_block(Block& b, uint64_t tiles, uint64_t aux) {
   CU(cudaMemset(b.sc.aux, 0, aux * 8));
   CU(cudaMemset(b.sc.aux2, 0, aux * 8));
   CU(cudaMemset(b.sc.aux3, 0, aux * 8));
+  CU(cudaMemset(b.sc.zacc, 0, aux * 8));
   CU(cudaMemset(b.sc.tbuf, 0, tiles * 8));
   CU(cudaMemset(b.sc.tbuf2, 0, tiles * 32));
   CU(cudaMemset(b.sc.tickets, 0, kEpochs * 4));
@@ -581,7 +584,7 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       zvc_compress_scratch(n, w, F, &tiles, &aux);
       Lease L(*c, st, tiles, aux);
       TRY(L.status);
-      c->launches += 2;  // accumulator zero fill + persistent compress
+      c->launches += 1;  // persistent compress (its accumulators clean up after themselves)
       const uint32_t ep = L.epoch();
       // per-frame publication from inside the persistent kernel only when asked (the D2H link
       // is idle, so the first frames' copies can overlap the rest of the compression); it costs
@@ -993,6 +996,7 @@ cswap_status cswap_shutdown(void) {
     cudaFree(b.sc.tbuf);
     cudaFree(b.sc.tbuf2);
     cudaFree(b.sc.aux3);
+    cudaFree(b.sc.zacc);
     cudaEventDestroy(b.ev);
   }
   cudaFree(c->dev_err);

@@ -38,6 +38,7 @@ struct Scratch {
   uint64_t* tbuf;         // per-tile u64 array for multi-kernel codecs (never epoch-tagged)
   uint64_t* tbuf2;        // second per-tile array, 32 bytes per tile (u64, or CSR: u32[8] slab counts)
   uint64_t* aux3;         // third per-frame u64 array (run / non-zero totals)
+  uint64_t* zacc;         // persistent ZVC compress accumulators (zero between launches; cap_aux)
   uint64_t cap_tiles, cap_aux;
   // swap-out progress (NULL outside cswap_swap_out): host-mapped pinned u64[K]; the compress
   // group stores kProgReady | (end offset of frame k in the container) once every byte of frame

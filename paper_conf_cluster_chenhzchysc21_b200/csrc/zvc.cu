@@ -214,7 +214,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     // acquire.cta), count it for its frame with a gpu-scope acq_rel atomic; the CTA that
     // completes a frame publishes the frame's end offset (frame start + its frame-table entry,
     // both written before the frame's last tiles were emitted) for the host's per-frame D2H
-    uint64_t* const fdone = sc.aux2 + K + uint64_t(K) * gpf;  // zeroed with the accumulators
+    uint64_t* const fdone = sc.zacc + K + uint64_t(K) * gpf;  // after the accumulators
     auto tile_emitted = [&](uint32_t t) {
       if (!sc.prog || lane != 0) return;
       uint32_t k, j, te, be;
@@ -278,10 +278,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       }
       if (done_t != SENT) tile_emitted(done_t);
     }
-    return;
-  }
-
-  if (warp > kProducerWarp) {  // -------------------------------- resolvers (one per stage)
+  } else if (warp > kProducerWarp) {  // ------------------------- resolvers (one per stage)
     const int r = warp - kProducerWarp - 1;
     for (uint32_t i = r;; i += S) {
       const int s = r;
@@ -312,7 +309,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           const uint64_t Fp = frame_len(n, F, k - 1);
           const uint64_t tiles_prev = cdiv(Fp, G::TILE);
           backoff = 32;
-          while (((acc = ld_relaxed(sc.aux2 + k - 1)) >> 40) != tiles_prev) {
+          while (((acc = ld_relaxed(sc.zacc + k - 1)) >> 40) != tiles_prev) {
             __nanosleep(backoff);
             backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
           }
@@ -327,7 +324,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           const uint32_t gi = g0 + lane;
           uint64_t v = 0;
           if (gi < g) {
-            const uint64_t* p = sc.aux2 + K + uint64_t(k) * gpf + gi;
+            const uint64_t* p = sc.zacc + K + uint64_t(k) * gpf + gi;
             uint32_t backoff = kMinBackoff;
             while (((v = ld_relaxed(p)) >> 40) != 32) {
               __nanosleep(backoff);
@@ -372,9 +369,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       __syncwarp();
       if (kNamedBars) named_arrive(kBarOff0 + s, 32 * (CW + 1));
     }
-    return;
-  }
-
+  } else {
   // ------------------------------------------------------------------------- consumers
   // CW warps, warp w owns slab w (PW elements = PW/32 rows of 32 words) of every tile.
   // count(i):   rows -> one ballot per row = one bitmap word (fp32) / two ballots (16-bit);
@@ -477,8 +472,8 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
 #pragma unroll
       for (int w = 0; w < CW; w++) tot += s_wtot[s][w];
       st_relaxed(sc.status + t, make_status(tot, epoch, kFlagA));  // self-contained: no release needed
-      atomicAdd(reinterpret_cast<unsigned long long*>(sc.aux2 + k), (1ull << 40) + tot);
-      atomicAdd(reinterpret_cast<unsigned long long*>(sc.aux2 + K + uint64_t(k) * gpf + j / 32), (1ull << 40) + tot);
+      atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + k), (1ull << 40) + tot);
+      atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + K + uint64_t(k) * gpf + j / 32), (1ull << 40) + tot);
       s_nnz[s] = tot;
       if (!kNamedBars) mbar_arrive(&bar_cnt[s]);
     }
@@ -563,6 +558,25 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     count(i, t);
     if (tid == 0) ZPROF_ADD(8, clock64() - c3);
     if (i >= uint32_t(LAG)) emit(i - LAG, s_ticket[(i - LAG) % S]);
+  }
+  }  // consumers
+
+  // The accumulators clean up after themselves (no zero-fill launch before the kernel): the
+  // last CTA to finish zeroes every accumulator word this launch used, so the next compress on
+  // this scratch block (stream-ordered after this one) starts from zeros.  sc.zacc is used by
+  // the persistent compress only; it is zeroed when the block is allocated.
+  __syncthreads();
+  __shared__ uint32_t s_last;
+  const uint64_t nacc = 2 * uint64_t(K) + uint64_t(K) * gpf;
+  if (tid == 0) {
+    unsigned long long old;
+    asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;" : "=l"(old) : "l"(sc.zacc + nacc) : "memory");
+    s_last = old + 1 == gridDim.x;
+  }
+  __syncthreads();
+  if (s_last) {
+    for (uint64_t q = tid; q < nacc; q += blockDim.x) sc.zacc[q] = 0;
+    if (tid == 0) sc.zacc[nacc] = 0;
   }
 }
 
@@ -884,9 +898,6 @@ static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uin
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, threads, L::bytes) != cudaSuccess || per_sm < 1)
       return cudaErrorInvalidConfiguration;
   }
-  // per-frame and per-group (tiles, nnz) accumulators
-  // (+ K per-frame emitted-tile counters for the swap-out progress words)
-  launch_zero_words(sc.aux2, (2 * uint64_t(K) + uint64_t(K) * ((tpf + 31) / 32)) * 2, st);
   const uint32_t cap = uint32_t(sm_count()) * uint32_t(per_sm);  // co-resident maximum
   const uint32_t want = g_zvc_grid.load(std::memory_order_relaxed);
   const uint32_t grid = std::min<uint32_t>(tiles, want ? std::min(want, cap) : cap);
@@ -970,7 +981,7 @@ static cudaError_t launch_compress_t(const void* in, uint64_t n, uint64_t F, uin
 void zvc_compress_scratch(uint64_t n, int w, uint64_t F, uint64_t* tiles, uint64_t* aux) {
   const uint64_t TILE = 16384 / w, K = cdiv(n, F), tpf = cdiv(F, TILE);
   *tiles = K ? (K - 1) * tpf + cdiv(frame_len(n, F, K - 1), TILE) : 0;
-  *aux = 2 * K + K * ((tpf + 31) / 32) + 2;
+  *aux = 2 * K + K * ((tpf + 31) / 32) + 2;  // sc.zacc: frame + group accumulators, fdone, CTA counter
 }
 
 cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,

@@ -63,8 +63,12 @@ class CSwapBackend:
         h.swap_in(out.view(-1), stream=stream)
 
     @staticmethod
+    def codec(h) -> int:
+        return h.codec()  # known when swap_out returns: no wait
+
+    @staticmethod
     def info(h) -> tuple[int, int]:
-        q = h.query()
+        q = h.query()  # waits until the swap-out's copies are issued
         return q["codec"], q["bytes"]
 
     @staticmethod
@@ -189,12 +193,15 @@ class SwapSaver:
         if self.verify:
             rec.original = t.detach().clone()
         rec.handle = self.backend.swap_out(t, codec, hf, hb)
-        rec.codec, rec.comp_bytes = self.backend.info(rec.handle)
+        # the codec is known at once; the container size only once the swap-out has run, so it is
+        # read when the record is released (reading it here would make every save wait for its
+        # compression, and the forward pass could no longer run ahead of the GPU)
+        rec.codec = self.backend.codec(rec.handle) if hasattr(self.backend, "codec") else \
+            self.backend.info(rec.handle)[0]
         self._live[key] = rec
         self._order.append(rec)
         self.stats["swapped"] += 1
         self.stats["raw_bytes"] += rec.nbytes
-        self.stats["comp_bytes"] += rec.comp_bytes
         self.stats["codecs"].append(rec.codec)
         return rec
 
@@ -226,6 +233,8 @@ class SwapSaver:
                 self.mismatches.append((rec.index, rec.codec))
         rec.refs -= 1
         if rec.refs == 0:  # every saving op has its copy: drop ours and the host container
+            rec.comp_bytes = self.backend.info(rec.handle)[1]
+            self.stats["comp_bytes"] += rec.comp_bytes
             rec.restored = None
             rec.original = None
             self.backend.free(rec.handle)

@@ -23,12 +23,18 @@ def main():
     ap.add_argument("--kind", default="iid", choices=["iid", "clustered"])
     ap.add_argument("--ncu", action="store_true")
     ap.add_argument("--check", action="store_true", help="verify round trip")
+    ap.add_argument("--variant", type=int, default=-1, help="ZVC compress geometry (cswap_set_zvc_launch)")
+    ap.add_argument("--grid", type=int, default=0, help="ZVC compress grid (0 = automatic)")
     a = ap.parse_args()
     import torch
 
     import synth
     from paper_conf_cluster_chenhzchysc21_b200 import cswap as C
     C.init(0)
+    C.set_zvc_launch(a.grid, a.variant)
+    sys.path.insert(0, ROOT)
+    from bench import ClockSampler
+    sampler = ClockSampler(0).__enter__()  # SM clock + throttle reasons under load (DESIGN §6 tables)
     names = {"none": C.NONE, "zvc": C.ZVC, "rle": C.RLE, "csr": C.CSR, "lz4": C.LZ4}
     dtype = {"f32": C.F32, "f16": C.F16, "bf16": C.BF16}[a.dtype]
     w = C.WIDTH[dtype]
@@ -60,7 +66,8 @@ def main():
             def decomp(nb):
                 C.decompress(buf, nb, y, n, dtype, codec, err=err)
 
-            res = {"codec": cname, "s": s, "MiB": a.mib, "dtype": a.dtype, "kind": a.kind}
+            res = {"codec": cname, "s": s, "MiB": a.mib, "dtype": a.dtype, "kind": a.kind,
+                   "variant": a.variant, "grid": a.grid}
             for label, fn in (("compress", comp), ("decompress", None)):
                 if fn is None:
                     nb = int(size.item())
@@ -91,6 +98,8 @@ def main():
             out.append(res)
             print(json.dumps(res), flush=True)
             del buf
+    sampler.__exit__(None, None, None)
+    print(json.dumps({"clocks": sampler.summary()}), flush=True)
     return out
 
 

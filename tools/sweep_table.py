@@ -1,4 +1,4 @@
-"""Markdown tables from a codec_bench JSONL sweep (tools/run_sweep.sh):
+"""Markdown tables from a codec_bench JSONL sweep (tools/gpu_tasks.sh sweep / zvc):
 per (kind, dtype, codec) rows of size x sparsity with compress / decompress fraction of the
 measured HBM peak (algorithmic bytes) and the compression ratio.
 
@@ -10,13 +10,20 @@ from collections import defaultdict
 
 
 def main():
-    rows = [json.loads(l) for l in open(sys.argv[1]) if l.strip().startswith("{")]
+    lines = [json.loads(l) for l in open(sys.argv[1]) if l.strip().startswith("{")]
+    rows = [r for r in lines if "codec" in r]
+    clocks = [r["clocks"] for r in lines if "clocks" in r]
     bad = [r for r in rows if r.get("roundtrip_ok") is False]
     groups = defaultdict(list)
     for r in rows:
         groups[(r.get("kind", "iid"), r["dtype"], r["codec"])].append(r)
     print(f"# Codec sweep ({len(rows)} points, round trips checked: "
           f"{sum(1 for r in rows if r.get('roundtrip_ok'))} ok, {len(bad)} failed)\n")
+    if clocks:
+        mhz = sorted(c["sm_mhz"] for c in clocks if c.get("sm_mhz"))
+        reasons = sorted({x for c in clocks for x in c.get("reasons", [])})
+        print(f"SM clock under load (nvidia-smi, {len(clocks)} runs): median {mhz[len(mhz) // 2] if mhz else None} MHz, "
+              f"max {clocks[0].get('sm_max_mhz')} MHz, throttle reasons {reasons or 'none'}\n")
     print("Cells: compress / decompress fraction of the measured HBM peak in algorithmic bytes "
           "(raw + container), ms in parentheses; ratio = container / raw.  tools/codec_bench.py, "
           "L2 flushed between reps, median.\n")
