@@ -177,6 +177,24 @@ cswap_status cswap_handle_query(const cswap_handle* h, cswap_codec* codec, uint6
                                 const void** host_container, cswap_decision* decision);
 void cswap_handle_free(cswap_handle* h);
 
+/* ---- swap target (NEXT-4b: peer HBM over NVLink, beyond the paper) ---------------------------- */
+/* Where cswap_swap_out puts containers from now on: -1 = pinned host memory (default; the paper's
+ * target); otherwise a CUDA device -- the device given to cswap_init (a
+ * container in local HBM) or a peer reachable by peer-to-peer access (NVLink 5 / NVSwitch on B200).
+ * With a device target the codec kernels store the container straight into that device's memory
+ * (peer-mapped stores, no host staging and no copy engine); swap-in decompresses straight from it.
+ * Containers of a device target have no host copy (cswap_handle_query's host_container = NULL;
+ * cswap_handle_copy_container reads them).  The selector keeps using the installed calibration:
+ * install one fitted for the peer link (cswap_set_calibration) when AUTO is used.
+ * Returns CSWAP_ERR_UNSUPPORTED if `device` cannot be reached by peer access, CSWAP_ERR_INVALID if
+ * it does not exist.  Handles already issued keep their own target. */
+cswap_status cswap_set_swap_target(int device);
+cswap_status cswap_get_swap_target(int* device);
+/* Copy h's container (container_bytes of cswap_handle_query, after its swap-out completed) into
+ * dst (host or device memory of at least `cap` bytes), ordered on `stream` and synchronised
+ * before returning.  Works for every target. */
+cswap_status cswap_handle_copy_container(cswap_handle* h, void* dst, uint64_t cap, void* stream);
+
 /* ---- calibration (a13) ----------------------------------------------------------------------- */
 /* Ordinary least squares t = b0 + b1*S + b2*S*s over m samples ("linear
  * regression"); beta_out[3].  Returns CSWAP_ERR_INVALID if m < 3 or the design is singular. */

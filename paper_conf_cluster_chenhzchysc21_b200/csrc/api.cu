@@ -174,6 +174,10 @@ struct Ctx {
   cudaStream_t s_d2h = nullptr, s_h2d = nullptr, s_h2d2 = nullptr;
   cudaMemPool_t pool = nullptr;  // private stream-ordered pool (staging, LZ4 slots, decode scratch)
   uint64_t* dev_sink = nullptr;  // device word for container sizes nobody reads
+  // swap target (cswap_set_swap_target): -1 = pinned host; else a device whose memory holds the
+  // containers (tpool: a pool located on that device, accessible from this one)
+  int target = -1;
+  cudaMemPool_t tpool = nullptr;
   // swap-out executor: one library thread turns published frames into D2H copies, FIFO
   std::thread exec;
   std::mutex qm;
@@ -722,6 +726,11 @@ struct cswap_handle {
   // executor's copy ranges; swap-in splits its H2D by these trusted values, never by the
   // host-resident frame table)
   std::vector<uint64_t> ends;
+  // device target (NEXT-4b): the container lives in device memory of `target` (no host copy);
+  // its size is written by the codec kernels into size_slot (pinned) and valid after ev_out
+  int target = -1;
+  uint8_t* dev = nullptr;
+  uint64_t* size_slot() { return reinterpret_cast<uint64_t*>(slots); }
 };
 
 namespace {
@@ -1002,6 +1011,7 @@ cswap_status cswap_shutdown(void) {
   cudaFree(c->dev_err);
   cudaFree(c->dev_sink);
   cudaMemPoolDestroy(c->pool);
+  if (c->tpool) cudaMemPoolDestroy(c->tpool);
   cudaStreamDestroy(c->s_d2h);
   cudaStreamDestroy(c->s_h2d);
   cudaStreamDestroy(c->s_h2d2);
@@ -1082,20 +1092,14 @@ cswap_status cswap_compress(const void* d_in, uint64_t n, cswap_dtype dtype, csw
                      static_cast<cudaStream_t>(stream));
 }
 
-cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uint64_t n, cswap_dtype dtype,
-                              cswap_codec codec, const cswap_format* fmt, uint32_t* err, void* stream) {
-  Ctx* c = nullptr;
-  TRY(need_ctx(&c));
+}  // extern "C"
+
+namespace {
+// decompress a whole container (device memory) into d_out on st; device-side validation
+// failures are merged into *user_err (device-visible word)
+cswap_status decompress_impl(Ctx* c, const uint8_t* inb, uint64_t in_size, void* d_out, uint64_t n, int dtype,
+                             int codec, const cswap_format& f, uint32_t* user_err, cudaStream_t st) {
   const int w = width(dtype);
-  if (!w) return fail(CSWAP_ERR_INVALID, "bad dtype %d", int(dtype));
-  if (codec > CSWAP_CODEC_LZ4) return fail(CSWAP_ERR_INVALID, "codec must be NONE/ZVC/RLE/CSR/LZ4");
-  TRY(check_common(in, "in"));
-  if (n) TRY(check_common(d_out, "d_out"));
-  if (in_size < 64) return fail(CSWAP_ERR_CORRUPT, "in_size < 64");
-  const cswap_format f = resolve_fmt(c, fmt);
-  TRY(check_fmt(f));
-  cudaStream_t st = static_cast<cudaStream_t>(stream);
-  uint32_t* user_err = err ? err : c->dev_err;
   const uint64_t F = f.frame_elems;
   const uint32_t K = uint32_t((n + F - 1) / F);
   Lease L(*c, st, decompress_tiles(n, w, f), decompress_aux(n, w, f));
@@ -1103,7 +1107,6 @@ cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uin
   // kernels flag errors in the lease's device word (never in host-mapped memory: every CTA
   // reads it); the word is merged into the caller's at the end
   uint32_t* e = L.b->sc.err;
-  const uint8_t* inb = static_cast<const uint8_t*>(in);
   uint8_t* tmp = nullptr;
   const uint64_t tmp_bytes = n ? decompress_tmp_bytes(codec, n, f, 0, K) : 0;
   if (tmp_bytes) CU(cudaMallocFromPoolAsync(reinterpret_cast<void**>(&tmp), tmp_bytes, c->pool, st));
@@ -1122,6 +1125,25 @@ cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uin
   });
   if (tmp) cudaFreeAsync(tmp, st);
   return s;
+}
+}  // namespace
+
+extern "C" {
+
+cswap_status cswap_decompress(const void* in, uint64_t in_size, void* d_out, uint64_t n, cswap_dtype dtype,
+                              cswap_codec codec, const cswap_format* fmt, uint32_t* err, void* stream) {
+  Ctx* c = nullptr;
+  TRY(need_ctx(&c));
+  const int w = width(dtype);
+  if (!w) return fail(CSWAP_ERR_INVALID, "bad dtype %d", int(dtype));
+  if (codec > CSWAP_CODEC_LZ4) return fail(CSWAP_ERR_INVALID, "codec must be NONE/ZVC/RLE/CSR/LZ4");
+  TRY(check_common(in, "in"));
+  if (n) TRY(check_common(d_out, "d_out"));
+  if (in_size < 64) return fail(CSWAP_ERR_CORRUPT, "in_size < 64");
+  const cswap_format f = resolve_fmt(c, fmt);
+  TRY(check_fmt(f));
+  return decompress_impl(c, static_cast<const uint8_t*>(in), in_size, d_out, n, dtype, codec, f,
+                         err ? err : c->dev_err, static_cast<cudaStream_t>(stream));
 }
 
 cswap_status cswap_check_device_error(void* stream) {
@@ -1207,6 +1229,59 @@ cswap_status cswap_select(const void* d_in, uint64_t n, cswap_dtype dtype, doubl
   return cswap_select_from_probe(n, dtype, &p, hidden_f, hidden_b, nullptr, out);
 }
 
+// ---- swap target (NEXT-4b) ------------------------------------------------------------------
+cswap_status cswap_set_swap_target(int device) {
+  Ctx* c = nullptr;
+  TRY(need_ctx(&c));
+  std::lock_guard<std::mutex> lk(c->cfg_m);
+  if (device < 0) {
+    c->target = -1;
+    return CSWAP_OK;
+  }
+  int count = 0;
+  CU(cudaGetDeviceCount(&count));
+  if (device >= count) return fail(CSWAP_ERR_INVALID, "device %d does not exist (%d visible)", device, count);
+  if (device != c->device) {
+    int ok = 0;
+    CU(cudaDeviceCanAccessPeer(&ok, c->device, device));
+    if (!ok) return fail(CSWAP_ERR_UNSUPPORTED, "device %d cannot reach device %d by peer access", c->device, device);
+    const cudaError_t e = cudaDeviceEnablePeerAccess(device, 0);
+    if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_status(e, "enable peer access");
+    cudaGetLastError();
+  }
+  if (c->tpool) {
+    cudaMemPoolDestroy(c->tpool);
+    c->tpool = nullptr;
+  }
+  // containers live in a pool located on the target device and accessible from this one: the
+  // codec kernels store into it (over NVLink for a peer) and the decoders read from it
+  cudaMemPoolProps pp = {};
+  pp.allocType = cudaMemAllocationTypePinned;
+  pp.location.type = cudaMemLocationTypeDevice;
+  pp.location.id = device;
+  CU(cudaMemPoolCreate(&c->tpool, &pp));
+  if (device != c->device) {
+    cudaMemAccessDesc ad = {};
+    ad.location.type = cudaMemLocationTypeDevice;
+    ad.location.id = c->device;
+    ad.flags = cudaMemAccessFlagsProtReadWrite;
+    CU(cudaMemPoolSetAccess(c->tpool, &ad, 1));
+  }
+  uint64_t keep = uint64_t(4096) << 20;
+  CU(cudaMemPoolSetAttribute(c->tpool, cudaMemPoolAttrReleaseThreshold, &keep));
+  c->target = device;
+  return CSWAP_OK;
+}
+
+cswap_status cswap_get_swap_target(int* device) {
+  Ctx* c = nullptr;
+  TRY(need_ctx(&c));
+  if (!device) return fail(CSWAP_ERR_INVALID, "device is NULL");
+  std::lock_guard<std::mutex> lk(c->cfg_m);
+  *device = c->target;
+  return CSWAP_OK;
+}
+
 // ---- swap pipeline ---------------------------------------------------------------------------
 cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, cswap_codec codec, double hidden_f,
                             double hidden_b, void* stream, cswap_handle** out) {
@@ -1255,6 +1330,36 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
   const uint64_t F = f.frame_elems;
   const uint32_t K = uint32_t((n + F - 1) / F);
   const uint64_t ds = al16(64 + 8ull * K);
+  cudaMemPool_t tpool = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(c->cfg_m);
+    h->target = c->target;
+    tpool = c->tpool;
+  }
+  if (h->target >= 0) {
+    // device target (NEXT-4b): the codec kernels write the container straight into the target's
+    // memory -- peer-mapped stores over NVLink for a peer -- sized for the codec's worst case;
+    // everything is ordered on the caller's stream, nothing waits on the host
+    const uint64_t cap = max_size(n, w, use, f);
+    if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&h->dev), cap, tpool, st) != cudaSuccess)
+      return bail(fail(CSWAP_ERR_NOMEM, "container of %llu B on device %d failed", (unsigned long long)cap, h->target));
+    h->cap = cap;
+    cswap_status s;
+    {
+      Timer tm(c, st);
+      s = do_compress(c, d_in, n, dtype, use, f, h->dev, h->size_slot(), st);
+      if (s == CSWAP_OK) tm.commit(use, 0, n * uint64_t(w), 0);
+    }
+    if (s == CSWAP_OK && cudaEventRecord(h->ev_out, st) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "event record");
+    if (s != CSWAP_OK) {
+      cudaFreeAsync(h->dev, st);
+      h->dev = nullptr;
+      return bail(s);
+    }
+    finish_out(h, 1, CSWAP_OK, "");
+    *out = h;
+    return CSWAP_OK;
+  }
   if (use == CSWAP_CODEC_NONE) {
     // raw offload (vDNN): the host writes header + frame table, the copy engine
     // moves the tensor's bytes straight into the frames after the caller's stream reaches here
@@ -1349,6 +1454,12 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
   const uint64_t ds = al16(64 + 8ull * K);
   h->in_issued = true;
   *h->err_slot() = 0;
+  if (h->dev) {  // device target: decode straight from the container (peer loads over NVLink)
+    CU(cudaStreamWaitEvent(st, h->ev_out, 0));  // same stream unless the caller switched streams
+    TRY(decompress_impl(c, h->dev, h->cap, d_out, n, h->dtype, h->codec, f, h->err_slot(), st));
+    CU(cudaEventRecord(h->ev_in, st));
+    return CSWAP_OK;
+  }
   if (n == 0) return cudaEventRecord(h->ev_in, st) == cudaSuccess ? CSWAP_OK : fail(CSWAP_ERR_CUDA, "record");
   if (h->ends.size() != K || h->ends.back() != h->bytes)
     return fail(CSWAP_ERR_CORRUPT, "frame ranges of the handle are inconsistent");
@@ -1476,6 +1587,10 @@ cswap_status cswap_handle_query(const cswap_handle* hc, cswap_codec* codec, uint
   if (decision) *decision = h->dec;
   if (container_bytes || host_container) {
     TRY(wait_out(h));
+    if (h->dev && !h->bytes) {  // device target: the size the codec kernels wrote
+      CU(cudaEventSynchronize(h->ev_out));
+      h->bytes = *reinterpret_cast<volatile uint64_t*>(h->size_slot());
+    }
     if (container_bytes) *container_bytes = h->bytes;
     if (host_container) *host_container = h->host;
   }
@@ -1489,9 +1604,22 @@ void cswap_handle_free(cswap_handle* h) {
   if (h->ev_in && h->in_issued) cudaEventSynchronize(h->ev_in);
   if (h->ev_out) cudaEventDestroy(h->ev_out);
   if (h->ev_in) cudaEventDestroy(h->ev_in);
+  if (h->dev) cudaFreeAsync(h->dev, h->ctx->s_d2h);  // every use is complete (events above)
   h->ctx->pinned.free(h->host);
   h->ctx->pinned.free(h->slots);
   delete h;
+}
+
+cswap_status cswap_handle_copy_container(cswap_handle* h, void* dst, uint64_t cap, void* stream) {
+  if (!h || !dst) return fail(CSWAP_ERR_INVALID, "bad arguments");
+  uint64_t bytes = 0;
+  TRY(cswap_handle_query(h, nullptr, &bytes, nullptr, nullptr));
+  if (cap < bytes) return fail(CSWAP_ERR_CAPACITY, "cap %llu < %llu", (unsigned long long)cap, (unsigned long long)bytes);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  CU(cudaStreamWaitEvent(st, h->ev_out, 0));
+  CU(cudaMemcpyAsync(dst, h->dev ? static_cast<const void*>(h->dev) : h->host, bytes, cudaMemcpyDefault, st));
+  CU(cudaStreamSynchronize(st));
+  return CSWAP_OK;
 }
 
 cswap_status cswap_fit_time_model(const double* S, const double* s, const double* t, uint64_t m, double* beta_out) {

@@ -109,6 +109,9 @@ _SIGS = {
     "cswap_kernel_launches": (_u64, []),
     "cswap_graph_stats": (None, [_P(_u64), _P(_u64)]),
     "cswap_set_zvc_launch": (_i, [_u32, ctypes.c_int32]),
+    "cswap_set_swap_target": (_i, [_i]),
+    "cswap_get_swap_target": (_i, [_P(ctypes.c_int)]),
+    "cswap_handle_copy_container": (_i, [_vp, _vp, _u64, _vp]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_L, _name)
@@ -259,6 +262,19 @@ class Handle:
                                      ctypes.byref(dec)), "cswap_handle_query")
         return {"codec": codec.value, "bytes": nbytes.value, "host": host.value, "decision": dec}
 
+    def copy_container(self, dst, cap: int, stream=None):
+        """Copy the container (any swap target) into dst (host or device, >= cap bytes)."""
+        _check(_L.cswap_handle_copy_container(self.raw, _ptr(dst), cap, _stream(stream)),
+               "cswap_handle_copy_container")
+
+    def container_bytes(self) -> bytes:
+        """The container's bytes, read through cswap_handle_copy_container (any target)."""
+        n = self.query()["bytes"]
+        buf = ctypes.create_string_buffer(max(n, 1))
+        if n:
+            self.copy_container(ctypes.addressof(buf), n)
+        return buf.raw[:n]
+
     def host_bytes(self) -> bytes:
         q = self.query()
         return ctypes.string_at(q["host"], q["bytes"]) if q["bytes"] else b""
@@ -273,6 +289,17 @@ class Handle:
             self.close()
         except Exception:
             pass
+
+
+def set_swap_target(device: int = -1):
+    """-1 = pinned host memory (default); else a device (this one or a peer over NVLink)."""
+    _check(_L.cswap_set_swap_target(device), "cswap_set_swap_target")
+
+
+def get_swap_target() -> int:
+    d = ctypes.c_int()
+    _check(_L.cswap_get_swap_target(ctypes.byref(d)), "cswap_get_swap_target")
+    return d.value
 
 
 def swap_out(d_in, n: int, dtype: int, codec: int = AUTO, hidden_f=0.0, hidden_b=0.0, stream=None) -> Handle:

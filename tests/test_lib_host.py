@@ -113,3 +113,13 @@ def test_max_size_matches_oracle(C, codec, dtype):
             param = {3: 512, 4: 2048}.get(codec, 0)
             fmt = (F, 512, 2048)
             assert C.max_compressed_size(n, dtype, codec, fmt) == O.max_size(codec, dtype, n, F, param)
+
+
+def test_swap_target_needs_init(C):
+    """cswap_set_swap_target (NEXT-4b) reports NOT_READY before cswap_init, like every call."""
+    with pytest.raises(C.CswapError) as e:
+        C.set_swap_target(1)
+    assert e.value.status == 7
+    with pytest.raises(C.CswapError) as e:
+        C.get_swap_target()
+    assert e.value.status == 7
