@@ -1167,36 +1167,44 @@ static cswap_status probe_impl(Ctx* c, const void* d_in, uint64_t n, int dtype, 
   if (n == 0) return CSWAP_OK;
   uint8_t* slot = c->pinned.alloc(256);
   if (!slot) return fail(CSWAP_ERR_NOMEM, "pinned alloc failed");
-  uint64_t* counts = reinterpret_cast<uint64_t*>(slot);
-  cudaEvent_t ev;
+  volatile uint64_t* counts = reinterpret_cast<volatile uint64_t*>(slot);
+  counts[0] = counts[1] = counts[2] = 0;
+  static std::atomic<uint32_t> tags{0};
+  uint32_t tag = 0;
+  while (tag == 0) tag = tags.fetch_add(1) & 0xFFFFu;  // nonzero, differs from the slot's last use
   cswap_status s = CSWAP_OK;
-  // spin-wait event: a blocking-sync event sleeps in the OS and wakes ~100 us late
-  if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) {
-    c->pinned.free(slot);
-    return fail(CSWAP_ERR_CUDA, "event create failed");
-  }
   {
     Lease L(*c, st, 1024, 1024);
     s = L.status;
     if (s == CSWAP_OK) {
       Timer tm(c, st);
       c->launches++;
-      s = cuda_status(launch_probe(d_in, n, w, counts, L.b->sc, L.epoch(), st), "probe");
+      s = cuda_status(launch_probe(d_in, n, w, reinterpret_cast<uint64_t*>(slot), tag, L.b->sc, L.epoch(), st),
+                      "probe");
       tm.commit(0, 2, std::min<uint64_t>(n, 262144) * w, 0);
     }
-    if (s == CSWAP_OK && cudaEventRecord(ev, st) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "event record");
   }
-  if (s == CSWAP_OK && cudaEventSynchronize(ev) != cudaSuccess) s = fail(CSWAP_ERR_CUDA, "probe sync failed");
+  // wait for the three tagged counts in mapped memory.  No completion event: an event record
+  // costs the stream ~25-35 us while a copy engine streams over PCIe (tools/event_probe.cu), the
+  // probe kernel itself ~7 us.  A failed or missing kernel is caught through the stream state.
+  auto ready = [&] { return (counts[0] & 0xFFFF) == tag && (counts[1] & 0xFFFF) == tag && (counts[2] & 0xFFFF) == tag; };
+  for (uint64_t spin = 0; s == CSWAP_OK && !ready(); spin++) {
+    if ((spin & 1023) == 1023) {
+      const cudaError_t e = cudaStreamQuery(st);
+      if (e == cudaSuccess && !ready()) s = fail(CSWAP_ERR_CUDA, "probe finished without publishing its counts");
+      else if (e != cudaSuccess && e != cudaErrorNotReady) s = cuda_status(e, "probe");
+    }
+    if (spin > 4096) std::this_thread::yield();
+  }
   if (s == CSWAP_OK) {
     const bool single = n <= 262144;
-    out->zeros = counts[0];
-    out->zero_runs = counts[1];
-    out->boundaries = counts[2];
+    out->zeros = counts[0] >> 16;
+    out->zero_runs = counts[1] >> 16;
+    out->boundaries = counts[2] >> 16;
     out->samples = single ? n : 262144;
     out->pairs = out->samples - (single ? 1 : 1024);
   }
-  cudaEventDestroy(ev);
-  c->pinned.free(slot);
+  if (s == CSWAP_OK) c->pinned.free(slot);  // (on failure the slot is leaked: the kernel may still write it)
   return s;
 }
 

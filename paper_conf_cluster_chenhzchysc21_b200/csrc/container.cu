@@ -244,7 +244,7 @@ constexpr int kProbeW = 256, kProbeSw = 1024;
 template <typename T>
 __global__ void __launch_bounds__(kThreads) probe_kernel(const T* __restrict__ x, uint64_t n, uint32_t pieces,
                                                          bool single, uint64_t* partial, uint32_t* done,
-                                                         uint64_t* counts3) {
+                                                         uint64_t* counts3, uint32_t tag) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   uint64_t z = 0, zr = 0, bd = 0;
   for (uint32_t p = blockIdx.x * kWarps + warp; p < pieces; p += gridDim.x * kWarps) {
@@ -291,22 +291,24 @@ __global__ void __launch_bounds__(kThreads) probe_kernel(const T* __restrict__ x
     uint64_t a = 0;
     for (uint32_t b = lane; b < gridDim.x; b += 32) a += __ldcg(partial + b * 3 + warp);
     a = warp_sum_u64(a);
-    if (lane == 0) counts3[warp] = a;
+    // one 64-bit store per count, tagged with this launch's 16-bit tag: the host polls the three
+    // words in mapped memory until all carry the tag (no completion event to wait for)
+    if (lane == 0) counts3[warp] = (a << 16) | tag;
   }
 }
 
-cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, const Scratch& sc, uint32_t epoch,
-                         cudaStream_t st) {
+cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, uint32_t tag, const Scratch& sc,
+                         uint32_t epoch, cudaStream_t st) {
   const bool single = n <= uint64_t(kProbeW) * kProbeSw;
   const uint32_t pieces = single ? uint32_t(cdiv(n, kProbeW)) : kProbeSw;
   const uint32_t grid = uint32_t(umin64(cdiv(pieces, kWarps), 128));
   timing_kernel_start(st);
   if (w == 4)
     probe_kernel<uint32_t><<<grid, kThreads, 0, st>>>(static_cast<const uint32_t*>(in), n, pieces, single, sc.aux2,
-                                                      sc.tickets + epoch, counts3);
+                                                      sc.tickets + epoch, counts3, tag);
   else
     probe_kernel<uint16_t><<<grid, kThreads, 0, st>>>(static_cast<const uint16_t*>(in), n, pieces, single, sc.aux2,
-                                                      sc.tickets + epoch, counts3);
+                                                      sc.tickets + epoch, counts3, tag);
   return cudaGetLastError();
 }
 

@@ -28,8 +28,9 @@ cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, 
                                  uint64_t* out_size, cudaStream_t st);
 cudaError_t launch_none_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, const Scratch& sc,
                                    uint32_t* err, cudaStream_t st);
-cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, const Scratch& sc, uint32_t epoch,
-                         cudaStream_t st);
+// counts3[c] = count << 16 | tag (host-mapped; the host polls for the tag)
+cudaError_t launch_probe(const void* in, uint64_t n, int w, uint64_t* counts3, uint32_t tag, const Scratch& sc,
+                         uint32_t epoch, cudaStream_t st);
 // swap-out progress of a finished compress group: prog[k] = kProgReady | end offset of frame k
 cudaError_t launch_publish_frames(const uint8_t* out, uint32_t K, uint64_t* prog, cudaStream_t st);
 

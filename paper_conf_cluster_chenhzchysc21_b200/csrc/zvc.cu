@@ -240,7 +240,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       uint32_t done_t = SENT;
       if (i >= S) {
         mbar_wait_sleep(&bar_empty[s], ((i / S) - 1) & 1, kProducerSleep);
-        done_t = s_ticket[s];
+        if (lane == 0) done_t = s_ticket[s];  // lane 0 alone reads and (below) rewrites the slot
       }
       if (lane == 0) ZPROF_ADD(0, clock64() - c0);
       // static round-robin assignment: CTA b takes tiles b, b + G, b + 2G, ... so every CTA
@@ -259,7 +259,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         if (sc.prog) {
           for (uint32_t p = i >= uint32_t(S - 1) ? i - (S - 1) : 0; p < i; p++) {
             mbar_wait_sleep(&bar_empty[p % S], (p / S) & 1, kProducerSleep);
-            tile_emitted(s_ticket[p % S]);
+            if (lane == 0) tile_emitted(s_ticket[p % S]);
           }
         }
         break;

@@ -20,7 +20,9 @@ def main():
     ap.add_argument("--s", default="0.5")
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--dtype", default="f32")
-    ap.add_argument("--kind", default="iid", choices=["iid", "clustered"])
+    ap.add_argument("--kind", default="iid", choices=["iid", "clustered", "clustered32", "dead", "zero", "dense"],
+                    help="zero placement (DESIGN.md §5): iid, clustered runs (mean zero run 256 / 32), "
+                         "channel-dead planes, all-zero, dense")
     ap.add_argument("--ncu", action="store_true")
     ap.add_argument("--check", action="store_true", help="verify round trip")
     ap.add_argument("--variant", type=int, default=-1, help="ZVC compress geometry (cswap_set_zvc_launch)")
@@ -44,11 +46,19 @@ def main():
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
     out = []
     for s in [float(v) for v in a.s.split(",")]:
+        import numpy as np
         if a.kind == "iid":
             x = synth.relu_iid_torch(n, s, seed=123, dtype=dtype, device="cuda")
+        elif a.kind == "dense":
+            x = synth.relu_iid_torch(n, 0.0, seed=123, dtype=dtype, device="cuda")
+        elif a.kind == "zero":
+            x = torch.zeros(n, dtype=torch.int32 if w == 4 else torch.int16, device="cuda")
+        elif a.kind == "dead":  # whole 56x56 planes of 64-channel images zero for a fraction s of the channels
+            hw = 56 * 56
+            h = synth.channel_dead((n // (64 * hw) + 1, 64, 56, 56), s, seed=7, dtype=dtype).reshape(-1)[:n]
+            x = torch.from_numpy(np.ascontiguousarray(h).view(np.int32 if w == 4 else np.int16)).cuda()
         else:
-            import numpy as np
-            h = synth.relu_clustered(n, s, 256, seed=5, dtype=dtype)
+            h = synth.relu_clustered(n, s, 256 if a.kind == "clustered" else 32, seed=5, dtype=dtype)
             x = torch.from_numpy(h.view(np.int32 if w == 4 else np.int16)).cuda()
         y = torch.empty_like(x)
         size = torch.zeros(1, dtype=torch.int64, device="cuda")

@@ -7,7 +7,8 @@
 #   bench      bench.py (VGG16 set, incl. extras) + BERT / ResNet-50 sets + the reference arm
 #   zvc        ZVC compress / decompress table: 1 GiB f32 / f16 / bf16 x s in {.2,.5,.8,.95}, and
 #              f32 / f16 at 16 / 24 / 96 / 256 MiB (codec_bench.py; L2 flushed; clocks recorded)
-#   sweep      BASELINE configs[1]: sizes x sparsities x 4 codecs, clustered, fp16 / bf16
+#   sweep      BASELINE configs[1]: sizes x sparsities x 4 codecs, clustered, fp16 / bf16 (+ sweep_kinds)
+#   sweep_kinds  clustered (L0 = 32), channel-dead, all-zero, dense at 64 MiB (appended to sweep.jsonl)
 #   profiles   ncu launch list of the bench command + ncu --set full summaries of the bench step's
 #              compress / decode launches and of the 1 GiB micro kernels (SASS mix, per-line)
 #   sanitize   compute-sanitizer memcheck / racecheck / synccheck / initcheck on tools/sanitize.py
@@ -43,7 +44,13 @@ for task in "$@"; do
     done; done
     for c in zvc rle csr lz4; do timeout 600 python tools/codec_bench.py --codecs $c --mib 64 --s 0.5,0.8,0.95,0.99 --kind clustered --check >> gpurun_out/sweep.jsonl 2>> gpurun_out/sweep.err; done
     for d in f16 bf16; do timeout 600 python tools/codec_bench.py --codecs zvc,rle,csr,lz4 --mib 64 --s 0.2,0.5,0.8 --dtype $d --check >> gpurun_out/sweep.jsonl 2>> gpurun_out/sweep.err; done
+    bash tools/gpu_tasks.sh sweep_kinds
     python tools/sweep_table.py gpurun_out/sweep.jsonl > gpurun_out/sweep.md 2>&1; wc -l gpurun_out/sweep.jsonl ;;
+  sweep_kinds)  # the other zero structures of SURVEY §8(d) at 64 MiB, appended to sweep.jsonl
+    for c in zvc rle csr lz4; do
+      for kind in clustered32 dead; do timeout 600 python tools/codec_bench.py --codecs $c --mib 64 --s 0.5,0.8,0.95,0.99 --kind $kind --check >> gpurun_out/sweep.jsonl 2>> gpurun_out/sweep.err; done
+      for kind in zero dense; do timeout 600 python tools/codec_bench.py --codecs $c --mib 64 --s 0.0 --kind $kind --check >> gpurun_out/sweep.jsonl 2>> gpurun_out/sweep.err; done
+    done ;;
   profiles)
     timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/p_launches.csv python bench.py --steps 2 --warmup 3 --no-extras --no-cpu > gpurun_out/p_launches.log 2>&1
     python tools/launch_summary.py gpurun_out/p_launches.csv "python bench.py --steps 2 --warmup 3 --no-extras --no-cpu (under ncu: warm-up + timed steps of the VGG16 b64 set, then the isolated replay of the 12 tensors x 4)" > gpurun_out/p_launches.txt
