@@ -171,15 +171,20 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         hs_last = None
+        marks = []  # an event at every step boundary: per-step times (steady state vs first steps)
         for i in range(steps):
             hs = step(codec)
             if i + 1 < steps:
+                marks.append(torch.cuda.Event(enable_timing=True))
+                marks[-1].record(stream)
                 for h in hs:
                     h.close()
             else:
                 hs_last = hs
         b.record(stream)
         b.synchronize()
+        bounds = [a] + marks + [b]
+        step_ms = [round(x.elapsed_time(y), 3) for x, y in zip(bounds, bounds[1:])]
         wall = time.perf_counter() - t0
         if sampler:
             sampler.__exit__(None, None, None)
@@ -193,7 +198,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
         for h in hs_last:
             h.close()
         return {"ms": ms, "wall_s": wall, "launches": launches, "records": recs, "handles": info,
-                "clocks": sampler.summary() if sampler else None}
+                "clocks": sampler.summary() if sampler else None, "step_ms": step_ms}
 
     # ---- headline: AUTO selection ---------------------------------------------------------
     main = timed(C.AUTO, args.steps, args.warmup, record=True, clocks=True)
@@ -216,6 +221,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
                    "l2": "working set 2.2 GB >> 126 MB L2: every step streams from HBM (no flush needed)",
                    "parallelism": f"replicas x{world}", "host_binding": numa},
         "gpu_launches": main["launches"],
+        "step_ms": main["step_ms"],
         "clocks": main["clocks"],
         "roofline": roof,
     }

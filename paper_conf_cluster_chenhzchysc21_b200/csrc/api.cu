@@ -95,7 +95,12 @@ struct PinnedPool {
         }
       }
     }
-    const uint64_t sz = std::max(bytes, chunk_bytes);
+    // new chunks grow geometrically (at least half of what is pinned already): pinning host
+    // memory costs milliseconds per GiB, so a workload reaches its steady footprint after a few
+    // allocations instead of pinning a chunk on every swap once the pool is fragmented
+    uint64_t pinned_total = 0;
+    for (auto& ch : chunks) pinned_total += ch.size;
+    const uint64_t sz = std::max({bytes, chunk_bytes, (pinned_total / 2 + 255) / 256 * 256});
     void* p = nullptr;
     if (cudaHostAlloc(&p, sz, cudaHostAllocPortable | cudaHostAllocMapped) != cudaSuccess) {
       cudaGetLastError();
@@ -741,6 +746,8 @@ struct OutJob {
   uint64_t* prog;    // host-mapped progress words (Scratch::prog)
   uint32_t K;
   cudaEvent_t done;  // recorded on the caller's stream after the compress group
+  bool exact_host;   // frames arrive all at once: allocate the host container at its exact size
+  uint64_t cap;      // staging bytes (the codec's worst case)
 };
 
 void finish_out(cswap_handle* h, int state, cswap_status err, const std::string& msg) {
@@ -821,7 +828,7 @@ void run_out_job(Ctx* c, OutJob* j) {
       const uint64_t v = prog[k_ready];
       if (!(v & kProgReady)) break;
       const uint64_t e = v & ~kProgReady;
-      if (e < (k_ready ? h->ends.back() : ds) || e > h->cap || (e & 15)) {
+      if (e < (k_ready ? h->ends.back() : ds) || e > j->cap || (e & 15)) {
         err = CSWAP_ERR_CUDA;
         msg = "inconsistent progress word from the compress kernel";
         break;
@@ -830,7 +837,18 @@ void run_out_job(Ctx* c, OutJob* j) {
       k_ready++;
     }
     if (err != CSWAP_OK) break;
-    if (k_ready > k) {
+    if (j->exact_host && k_ready == j->K && !h->host) {
+      // every frame is published at once (publication after the codec's last kernel): pin the
+      // container at its exact size (no worst-case allocation: RLE / CSR reserve 2-3x raw)
+      h->host = c->pinned.alloc(h->ends.back());
+      h->cap = h->ends.back();
+      if (!h->host) {
+        err = CSWAP_ERR_NOMEM;
+        msg = "pinned alloc of the container failed";
+        break;
+      }
+    }
+    if (k_ready > k && (!j->exact_host || k_ready == j->K)) {  // exact_host: the whole container at once
       const uint64_t end = h->ends[k_ready - 1];
       // copy granularity: a D2H copy costs a few us of DMA ramp and tail (8 MiB copies ran at
       // 52.2 GB/s, whole tensors at 54.0, tools/pipeline_probe.py), so published frames are
@@ -871,6 +889,14 @@ void run_out_job(Ctx* c, OutJob* j) {
     // then back off so that a long queue of pending compresses does not burn a core
     if (++idle < 4096) std::this_thread::yield();
     else std::this_thread::sleep_for(std::chrono::microseconds(20));
+  }
+  if (err == CSWAP_OK && !h->host) {  // n = 0: a header-only container
+    h->host = c->pinned.alloc(pos);
+    h->cap = pos;
+    if (!h->host) {
+      err = CSWAP_ERR_NOMEM;
+      msg = "pinned alloc of the container failed";
+    }
   }
   if (err == CSWAP_OK) write_host_header(h);
   // staging is freed on the D2H stream behind the copies; when nothing waited for the kernels
@@ -964,14 +990,16 @@ cswap_status cswap_init(int device) {
     TRY(ensure_block(b, 1 << 16, 1 << 12));
   }
   // a private pool ("memory pool"): staging memory stays reserved between swaps up
-  // to a bounded threshold (CSWAP_POOL_KEEP_MB, default 4096) and the process's default pool is
-  // left as the application configured it
+  // to a bounded threshold (CSWAP_POOL_KEEP_MB, default 16 GiB of the 180: a training step's
+  // worst-case staging in flight; trimming below it made every step re-map pool memory, which
+  // stalled the forward pass) and the process's default pool is left as the
+  // application configured it
   cudaMemPoolProps pp = {};
   pp.allocType = cudaMemAllocationTypePinned;
   pp.location.type = cudaMemLocationTypeDevice;
   pp.location.id = device;
   CU(cudaMemPoolCreate(&c->pool, &pp));
-  uint64_t keep = uint64_t(4096) << 20;
+  uint64_t keep = uint64_t(16384) << 20;
   if (const char* e = getenv("CSWAP_POOL_KEEP_MB")) keep = uint64_t(atoll(e)) << 20;
   CU(cudaMemPoolSetAttribute(c->pool, cudaMemPoolAttrReleaseThreshold, &keep));
   CU(cudaMalloc(&c->dev_err, 64));
@@ -1406,10 +1434,24 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
   uint8_t* staging = nullptr;
   if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging), cap, c->pool, st) != cudaSuccess)
     return bail(fail(CSWAP_ERR_NOMEM, "device staging of %llu B failed", (unsigned long long)cap));
-  h->host = c->pinned.alloc(cap);
-  h->cap = cap;
+  // per-frame publication pays only when the D2H link would otherwise wait for this tensor's
+  // compression (nothing queued ahead of it); CSWAP_FRAME_PUBLISH=0/1 forces it off/on.  Only
+  // ZVC publishes from inside its kernel; then the host container is pinned at the worst case
+  // (1.03x raw) up front, else the executor pins it at its exact size once it is known.
+  bool frame_publish;
+  if (const char* e = getenv("CSWAP_FRAME_PUBLISH")) {
+    frame_publish = e[0] == '1';
+  } else {
+    std::lock_guard<std::mutex> lk(c->qm);
+    frame_publish = c->q.empty() && cudaStreamQuery(c->s_d2h) == cudaSuccess;
+  }
+  frame_publish = frame_publish && use == CSWAP_CODEC_ZVC;
+  if (frame_publish) {
+    h->host = c->pinned.alloc(cap);
+    h->cap = cap;
+  }
   uint64_t* prog = reinterpret_cast<uint64_t*>(c->pinned.alloc(8ull * std::max<uint32_t>(K, 1)));
-  if (!h->host || !prog) {
+  if ((frame_publish && !h->host) || !prog) {
     cudaFreeAsync(staging, st);
     c->pinned.free(reinterpret_cast<uint8_t*>(prog));
     return bail(fail(CSWAP_ERR_NOMEM, "pinned alloc of %llu B failed", (unsigned long long)cap));
@@ -1422,15 +1464,6 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     // the container size goes to the timer's pinned slot when timing (read at collection), else
     // to a device word nobody reads (the executor takes the size from the progress words)
     uint64_t* osz = tm.stamps ? tm.stamps + 2 : c->dev_sink;
-    // per-frame publication pays only when the D2H link would otherwise wait for this tensor's
-    // compression (nothing queued ahead of it); CSWAP_FRAME_PUBLISH=0/1 forces it off/on
-    bool frame_publish;
-    if (const char* e = getenv("CSWAP_FRAME_PUBLISH")) {
-      frame_publish = e[0] == '1';
-    } else {
-      std::lock_guard<std::mutex> lk(c->qm);
-      frame_publish = c->q.empty() && cudaStreamQuery(c->s_d2h) == cudaSuccess;
-    }
     s = do_compress(c, d_in, n, dtype, use, f, staging, osz, st, prog, frame_publish);
     if (s == CSWAP_OK) tm.commit(use, 0, n * uint64_t(w), 0);
   }
@@ -1444,7 +1477,7 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     c->pinned.free(reinterpret_cast<uint8_t*>(prog));
     return bail(s);
   }
-  enqueue_out(c, new OutJob{h, staging, prog, K, done});
+  enqueue_out(c, new OutJob{h, staging, prog, K, done, !frame_publish, cap});
   *out = h;
   return CSWAP_OK;
 }
