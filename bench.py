@@ -588,15 +588,21 @@ def _e2e(args, C, torch, tensors, outs, sizes, dtype, w, dist, world, stream) ->
         dist.barrier()
     a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     a.record(stream)
-    for _ in range(steps):
+    marks = []
+    for i in range(steps):
         for h in one():
             h.close()
+        if i + 1 < steps:
+            marks.append(torch.cuda.Event(enable_timing=True))
+            marks[-1].record(stream)
     b.record(stream)
     b.synchronize()
+    bounds = [a] + marks + [b]
+    step_ms = [round(x.elapsed_time(y), 3) for x, y in zip(bounds, bounds[1:])]
     ms = _max_over_ranks(a.elapsed_time(b), dist) / steps
     raw = sum(sizes) * w
     return {"value": round(world * raw / (ms * 1e-3) / 1e9, 3), "unit": "GB/s", "ms_per_step": round(ms, 3),
-            "h2d_bytes_per_step": raw, "d2h_bytes_per_step": 16 * len(tensors), "steps": steps}
+            "h2d_bytes_per_step": raw, "d2h_bytes_per_step": 16 * len(tensors), "steps": steps, "step_ms": step_ms}
 
 
 def _cpu_model() -> str:

@@ -79,9 +79,7 @@ struct PinnedPool {
 
   static uint64_t round(uint64_t b) { return std::max<uint64_t>(256, (b + 255) / 256 * 256); }
 
-  uint8_t* alloc(uint64_t bytes) {
-    bytes = round(bytes);
-    std::lock_guard<std::mutex> lk(m);
+  uint8_t* take(uint64_t bytes) {  // first fit; caller holds m
     for (size_t c = 0; c < chunks.size(); c++) {
       auto& fl = chunks[c].free;
       for (auto it = fl.begin(); it != fl.end(); ++it) {
@@ -95,21 +93,30 @@ struct PinnedPool {
         }
       }
     }
+    return nullptr;
+  }
+  uint8_t* alloc(uint64_t bytes) {
+    bytes = round(bytes);
+    uint64_t pinned_total = 0;
+    {
+      std::lock_guard<std::mutex> lk(m);
+      if (uint8_t* p = take(bytes)) return p;
+      for (auto& ch : chunks) pinned_total += ch.size;
+    }
     // new chunks grow geometrically (at least half of what is pinned already): pinning host
     // memory costs milliseconds per GiB, so a workload reaches its steady footprint after a few
-    // allocations instead of pinning a chunk on every swap once the pool is fragmented
-    uint64_t pinned_total = 0;
-    for (auto& ch : chunks) pinned_total += ch.size;
+    // allocations instead of pinning a chunk on every swap once the pool is fragmented.  The
+    // pinning runs outside the lock, so other threads' allocations are not held behind it.
     const uint64_t sz = std::max({bytes, chunk_bytes, (pinned_total / 2 + 255) / 256 * 256});
     void* p = nullptr;
     if (cudaHostAlloc(&p, sz, cudaHostAllocPortable | cudaHostAllocMapped) != cudaSuccess) {
       cudaGetLastError();
       return nullptr;
     }
+    std::lock_guard<std::mutex> lk(m);
     chunks.push_back(Chunk{static_cast<uint8_t*>(p), sz, {}});
-    if (sz > bytes) chunks.back().free[bytes] = sz - bytes;
-    live[static_cast<uint8_t*>(p)] = {chunks.size() - 1, bytes};
-    return static_cast<uint8_t*>(p);
+    chunks.back().free[0] = sz;
+    return take(bytes);
   }
   void release_range(size_t c, uint64_t off, uint64_t bytes) {
     auto& fl = chunks[c].free;
@@ -193,7 +200,8 @@ struct Ctx {
   std::mutex cfg_m;
   cswap_calib calib{};
   cswap_format fmt{};
-  PinnedPool pinned;
+  PinnedPool pinned;  // host containers
+  PinnedPool small;   // progress words, probe counts, timer stamps, handle slots (never wait on a container's pinning)
   uint32_t* dev_err = nullptr;  // err word for cswap_decompress(err = NULL)
   std::atomic<uint64_t> launches{0};
   std::atomic<uint64_t> graph_launches{0}, graph_instantiations{0};
@@ -250,7 +258,7 @@ namespace {
 Timer::Timer(Ctx* ctx, cudaStream_t s) : c(ctx), st(s) {
   if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) {
     t_pending = this;
-    stamps = reinterpret_cast<uint64_t*>(c->pinned.alloc(24));
+    stamps = reinterpret_cast<uint64_t*>(c->small.alloc(24));
     if (stamps) stamps[0] = stamps[1] = stamps[2] = 0;
   }
 }
@@ -258,7 +266,7 @@ Timer::~Timer() {
   if (t_pending == this) t_pending = nullptr;
   if (a) cudaEventDestroy(a);
   if (b) cudaEventDestroy(b);
-  if (stamps) c->pinned.free(reinterpret_cast<uint8_t*>(stamps));  // not committed
+  if (stamps) c->small.free(reinterpret_cast<uint8_t*>(stamps));  // not committed
 }
 }  // namespace
 
@@ -905,7 +913,7 @@ void run_out_job(Ctx* c, OutJob* j) {
   cudaFreeAsync(j->staging, c->s_d2h);
   cudaEventRecord(h->ev_out, c->s_d2h);
   cudaEventDestroy(j->done);
-  c->pinned.free(reinterpret_cast<uint8_t*>(j->prog));  // the kernel has written its last word
+  c->small.free(reinterpret_cast<uint8_t*>(j->prog));  // the kernel has written its last word
   if (err == CSWAP_OK) {
     h->bytes = pos;
     c->pinned.shrink(h->host, pos);
@@ -1006,6 +1014,7 @@ cswap_status cswap_init(int device) {
   CU(cudaMemset(c->dev_err, 0, 64));
   CU(cudaMalloc(&c->dev_sink, 64));
   if (const char* e = getenv("CSWAP_PINNED_CHUNK_MB")) c->pinned.chunk_bytes = uint64_t(atoll(e)) << 20;
+  c->small.chunk_bytes = uint64_t(1) << 20;
   c->calib = builtin_calib();
   c->fmt = cswap_format{uint64_t(1) << 22, 1024, 65536};
   c->exec = std::thread(executor_main, c);
@@ -1044,6 +1053,7 @@ cswap_status cswap_shutdown(void) {
   cudaStreamDestroy(c->s_h2d);
   cudaStreamDestroy(c->s_h2d2);
   c->pinned.destroy();
+  c->small.destroy();
   delete c;
   g_ctx = nullptr;
   return CSWAP_OK;
@@ -1193,7 +1203,7 @@ static cswap_status probe_impl(Ctx* c, const void* d_in, uint64_t n, int dtype, 
   const int w = width(dtype);
   std::memset(out, 0, sizeof(*out));
   if (n == 0) return CSWAP_OK;
-  uint8_t* slot = c->pinned.alloc(256);
+  uint8_t* slot = c->small.alloc(256);
   if (!slot) return fail(CSWAP_ERR_NOMEM, "pinned alloc failed");
   volatile uint64_t* counts = reinterpret_cast<volatile uint64_t*>(slot);
   counts[0] = counts[1] = counts[2] = 0;
@@ -1232,7 +1242,7 @@ static cswap_status probe_impl(Ctx* c, const void* d_in, uint64_t n, int dtype, 
     out->samples = single ? n : 262144;
     out->pairs = out->samples - (single ? 1 : 1024);
   }
-  if (s == CSWAP_OK) c->pinned.free(slot);  // (on failure the slot is leaked: the kernel may still write it)
+  if (s == CSWAP_OK) c->small.free(slot);  // (on failure the slot is leaked: the kernel may still write it)
   return s;
 }
 
@@ -1334,7 +1344,7 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
   h->n = n;
   h->dtype = dtype;
   h->fmt = f;
-  h->slots = c->pinned.alloc(256);
+  h->slots = c->small.alloc(256);
   if (!h->slots) {
     delete h;
     return fail(CSWAP_ERR_NOMEM, "pinned alloc failed");
@@ -1450,10 +1460,10 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     h->host = c->pinned.alloc(cap);
     h->cap = cap;
   }
-  uint64_t* prog = reinterpret_cast<uint64_t*>(c->pinned.alloc(8ull * std::max<uint32_t>(K, 1)));
+  uint64_t* prog = reinterpret_cast<uint64_t*>(c->small.alloc(8ull * std::max<uint32_t>(K, 1)));
   if ((frame_publish && !h->host) || !prog) {
     cudaFreeAsync(staging, st);
-    c->pinned.free(reinterpret_cast<uint8_t*>(prog));
+    c->small.free(reinterpret_cast<uint8_t*>(prog));
     return bail(fail(CSWAP_ERR_NOMEM, "pinned alloc of %llu B failed", (unsigned long long)cap));
   }
   std::memset(prog, 0, 8ull * std::max<uint32_t>(K, 1));
@@ -1474,7 +1484,7 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     if (done) cudaEventDestroy(done);
     cudaFreeAsync(staging, st);
     cudaStreamSynchronize(st);  // the group may have been partly enqueued: prog is still referenced
-    c->pinned.free(reinterpret_cast<uint8_t*>(prog));
+    c->small.free(reinterpret_cast<uint8_t*>(prog));
     return bail(s);
   }
   enqueue_out(c, new OutJob{h, staging, prog, K, done, !frame_publish, cap});
@@ -1535,6 +1545,7 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
   // decode launch group each; a copy's DMA ramp / tail costs a few us, so the link runs at
   // 53.4 GB/s with one copy per 8 MiB frame and 54.7 with ~32 MiB copies)
   const uint64_t min_group = env_bytes("CSWAP_SWAPIN_GROUP_MB", uint64_t(32) << 20);
+  const bool two_streams = !(getenv("CSWAP_SWAPIN_STREAMS") && getenv("CSWAP_SWAPIN_STREAMS")[0] == '1');
   std::vector<uint32_t> gk{0};
   {
     uint64_t start = 0;
@@ -1557,7 +1568,7 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
         s = fail(CSWAP_ERR_CORRUPT, "frame range out of bounds");
         break;
       }
-      cudaStream_t cs = (gi & 1) ? c->s_h2d2 : c->s_h2d;
+      cudaStream_t cs = ((gi & 1) && two_streams) ? c->s_h2d2 : c->s_h2d;
       cudaEvent_t e;
       if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) {
         s = fail(CSWAP_ERR_CUDA, "event create");
@@ -1647,7 +1658,7 @@ void cswap_handle_free(cswap_handle* h) {
   if (h->ev_in) cudaEventDestroy(h->ev_in);
   if (h->dev) cudaFreeAsync(h->dev, h->ctx->s_d2h);  // every use is complete (events above)
   h->ctx->pinned.free(h->host);
-  h->ctx->pinned.free(h->slots);
+  h->ctx->small.free(h->slots);
   delete h;
 }
 
@@ -1700,7 +1711,7 @@ uint64_t cswap_collect_kernel_timing(cswap_kernel_record* out, uint64_t cap) {
       const volatile uint64_t* t = e.stamps;
       e.r.device_ms = (t[0] && t[1] > t[0]) ? double(t[1] - t[0]) * 1e-6 : 0.0;
       if (!e.r.comp_bytes) e.r.comp_bytes = t[2];  // swap-out compress: container size
-      c->pinned.free(reinterpret_cast<uint8_t*>(e.stamps));
+      c->small.free(reinterpret_cast<uint8_t*>(e.stamps));
     }
     if (out && k < cap) out[k] = e.r;
     k++;
