@@ -29,7 +29,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "compressed swap-out+in latency & codec GB/s vs HBM roofline, 1/2/4/8 B200"
 CALIB_PATH = os.path.join(ROOT, "calib", "b200.json")
-NCU_SUMMARY = os.path.join(ROOT, "profiles", "ncu_r01.json")
+NCU_SUMMARY = os.path.join(ROOT, "profiles", "ncu_r02.json")
 
 
 def log(*a):
@@ -121,6 +121,10 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
     torch.cuda.set_device(local_rank)
     numa = _bind_local_cpus(local_rank)
     C.init(local_rank)  # the pinned pools are first-touched by this (now GPU-local) thread
+    if args.swap_target != "host":
+        if args.swap_target == "peer" and world < 2:
+            raise SystemExit("bench.py: --swap-target peer needs --gpus >= 2")
+        C.set_swap_target(local_rank if args.swap_target == "self" else (local_rank + 1) % world)
     codecs_built = [c for c in (C.ZVC, C.RLE, C.CSR, C.LZ4) if _codec_built(C, c)]
     if args.calibrate or not calibrate.load(CALIB_PATH):
         log(f"calibrating on the box (codecs {codecs_built}) ...")
@@ -219,7 +223,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
                    "elem": synth.NAMES[dtype], "selector": "pipelined" if cal.mode == 0 else "paper",
                    "frame_elems": int(C.get_format().frame_elems),
                    "l2": "working set 2.2 GB >> 126 MB L2: every step streams from HBM (no flush needed)",
-                   "parallelism": f"replicas x{world}", "host_binding": numa},
+                   "parallelism": f"replicas x{world}", "host_binding": numa, "swap_target": args.swap_target},
         "gpu_launches": main["launches"],
         "step_ms": main["step_ms"],
         "clocks": main["clocks"],
@@ -476,6 +480,29 @@ def _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, r
         tp.append((t1 - t0, t2 - t1))
     ex["overheads_us"] = {"probe_incl_readback": round(1e6 * sum(a for a, _ in tp) / len(tp), 2),
                           "select_host": round(1e6 * sum(b for _, b in tp) / len(tp), 2)}
+    # host time of a fixed-codec swap-out call while the stream is busy (it only enqueues: no
+    # device wait), for the largest tensor of the set; a no-op call through the same binding
+    # gives the Python / ctypes share
+    big = max(range(len(tensors)), key=lambda i: sizes[i])
+    for h in [C.swap_out(tensors[big], sizes[big], dtype, C.ZVC) for _ in range(2)]:
+        h.close()
+    torch.cuda.synchronize()
+    torch.cuda._sleep(200_000_000)
+    hs, th = [], []
+    for _ in range(10):
+        t0 = time.perf_counter()
+        hs.append(C.swap_out(tensors[big], sizes[big], dtype, C.ZVC))
+        th.append(time.perf_counter() - t0)
+    t_noop = []
+    for _ in range(10):
+        t0 = time.perf_counter()
+        C.kernel_launches()
+        t_noop.append(time.perf_counter() - t0)
+    for h in hs:
+        h.close()
+    ex["overheads_us"]["swap_out_call_busy_stream"] = {
+        "tensor_MiB": sizes[big] * w / 2**20, "median_us": round(1e6 * statistics.median(th), 1),
+        "min_us": round(1e6 * min(th), 1), "noop_binding_call_us": round(1e6 * statistics.median(t_noop), 1)}
     return ex
 
 
@@ -824,6 +851,9 @@ def main(argv=None):
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--stub", action="store_true", help=argparse.SUPPRESS)  # CPU test of the launcher
+    ap.add_argument("--swap-target", default="host", choices=["host", "peer", "self"],
+                    help="where containers go (NEXT-4b): pinned host memory, the next GPU's HBM over NVLink "
+                         "(rank r -> (r + 1) mod N), or this GPU's HBM")
     ap.add_argument("--cpu-plan", metavar="OUT_JSON", help="oracle timing plan of SURVEY §8(d) (CPU only)")
     args = ap.parse_args(argv)
     if args.cpu_plan:

@@ -98,6 +98,23 @@ constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
 #endif
 constexpr uint32_t kProducerSleep = 256 * CSWAP_ZVC_SLEEP, kResolverSleep = 128 * CSWAP_ZVC_SLEEP,
                    kConsumerSleep = 64 * CSWAP_ZVC_SLEEP;
+// how the producer (bar_empty) and the consumers' polling warp (bar_full) wait: 0 = test +
+// __nanosleep backoff, 1 = mbarrier.try_wait, which suspends the warp in hardware until the phase
+// completes or ~4 us pass (tools/sleep_probe.cu: one instruction per wake-up instead of one poll
+// per 66-513 ns of __nanosleep).  A/B at 1 GiB f32 / f16 and 96 MiB: the same times within the
+// event timer's 2 us steps (the kernel is latency-bound in the consumers, not issue-bound), so
+// 1 is kept for the issue slots it leaves to kernels sharing the SMs
+
+#ifndef CSWAP_ZVC_PWAIT
+#define CSWAP_ZVC_PWAIT 1
+#endif
+#ifndef CSWAP_ZVC_CWAIT
+#define CSWAP_ZVC_CWAIT 1
+#endif
+__device__ __forceinline__ void producer_wait(uint64_t* bar, uint32_t parity) {
+  if (CSWAP_ZVC_PWAIT) mbar_wait(bar, parity);
+  else mbar_wait_sleep(bar, parity, kProducerSleep);
+}
 
 // the resolver handshakes (tile counted -> resolver; offset resolved -> consumers) on named
 // barriers (bar.arrive / bar.sync: a waiting warp issues nothing) instead of polled mbarriers
@@ -239,7 +256,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       // the stage is refilled, so the atomic's round trip never delays the next TMA load
       uint32_t done_t = SENT;
       if (i >= S) {
-        mbar_wait_sleep(&bar_empty[s], ((i / S) - 1) & 1, kProducerSleep);
+        producer_wait(&bar_empty[s], ((i / S) - 1) & 1);
         if (lane == 0) done_t = s_ticket[s];  // lane 0 alone reads and (below) rewrites the slot
       }
       if (lane == 0) ZPROF_ADD(0, clock64() - c0);
@@ -258,7 +275,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         // the tiles of rounds i-S+1 .. i-1 are still being emitted: wait for each and count it
         if (sc.prog) {
           for (uint32_t p = i >= uint32_t(S - 1) ? i - (S - 1) : 0; p < i; p++) {
-            mbar_wait_sleep(&bar_empty[p % S], (p / S) & 1, kProducerSleep);
+            producer_wait(&bar_empty[p % S], (p / S) & 1);
             if (lane == 0) tile_emitted(s_ticket[p % S]);
           }
         }
@@ -388,7 +405,10 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
   };
   constexpr int EROWS = PW / 32;  // rows of 32 elements per slab
   auto group_wait = [&](uint64_t* bar, uint32_t parity) {  // one warp polls, the rest block in bar.sync
-    if (warp == 0) mbar_wait_sleep(bar, parity, kConsumerSleep);
+    if (warp == 0) {
+      if (CSWAP_ZVC_CWAIT) mbar_wait(bar, parity);
+      else mbar_wait_sleep(bar, parity, kConsumerSleep);
+    }
     consumer_sync();
     if (warp != 0) mbar_wait(bar, parity);  // phase already complete: returns at once
   };
