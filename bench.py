@@ -484,15 +484,17 @@ def _extras(args, C, torch, tensors, outs, sizes, dtype, w, timed, main, dist, r
     # device wait), for the largest tensor of the set; a no-op call through the same binding
     # gives the Python / ctypes share
     big = max(range(len(tensors)), key=lambda i: sizes[i])
-    for h in [C.swap_out(tensors[big], sizes[big], dtype, C.ZVC) for _ in range(2)]:
-        h.close()
-    torch.cuda.synchronize()
-    torch.cuda._sleep(200_000_000)
-    hs, th = [], []
-    for _ in range(10):
-        t0 = time.perf_counter()
-        hs.append(C.swap_out(tensors[big], sizes[big], dtype, C.ZVC))
-        th.append(time.perf_counter() - t0)
+    for rep in range(2):  # the first pass grows the staging / pinned pools to 10 outstanding swaps
+        torch.cuda.synchronize()
+        torch.cuda._sleep(200_000_000)
+        hs, th = [], []
+        for _ in range(10):
+            t0 = time.perf_counter()
+            hs.append(C.swap_out(tensors[big], sizes[big], dtype, C.ZVC))
+            th.append(time.perf_counter() - t0)
+        if rep == 0:
+            for h in hs:
+                h.close()
     t_noop = []
     for _ in range(10):
         t0 = time.perf_counter()

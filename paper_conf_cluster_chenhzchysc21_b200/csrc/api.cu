@@ -838,7 +838,13 @@ void run_out_job(Ctx* c, OutJob* j) {
       const uint64_t e = v & ~kProgReady;
       if (e < (k_ready ? h->ends.back() : ds) || e > j->cap || (e & 15)) {
         err = CSWAP_ERR_CUDA;
-        msg = "inconsistent progress word from the compress kernel";
+        char b[256];
+        snprintf(b, sizeof(b),
+                 "inconsistent progress word from the compress kernel (codec %d, frame %u of %u: end %llu, "
+                 "previous %llu, capacity %llu)",
+                 h->codec, k_ready, j->K, (unsigned long long)e,
+                 (unsigned long long)(k_ready ? h->ends.back() : ds), (unsigned long long)j->cap);
+        msg = b;
         break;
       }
       h->ends.push_back(e);

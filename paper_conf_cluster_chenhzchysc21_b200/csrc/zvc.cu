@@ -534,8 +534,6 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         if (uint32_t(lane) < nv) stg_stream(bdst + lane, bsrc[lane]);
       }
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&bar_empty[s]);  // this warp no longer reads the stage
     const uint64_t g1 = g0 + uint64_t(nnz) * G::W;
     if (warp == CW - 1 && lane == 31) {
       if (uint64_t(j) * G::TILE + G::TILE >= Fk) {  // last tile of the frame: pad + frame_bytes[k]
@@ -549,6 +547,11 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         *out_size = total;
       }
     }
+    // the stage is released only after every store of this warp's part of the tile, the frame's
+    // pad and frame-table entry included: the producer counts the tile as emitted on this
+    // barrier and may then publish the frame (swap-out progress) with that entry
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&bar_empty[s]);
     if (tid == 0) ZPROF_ADD(6, clock64() - c2);
   };
 
