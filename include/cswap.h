@@ -119,8 +119,9 @@ cswap_status cswap_get_format(cswap_format* out);
  * (0: 3 x 32 KiB stages, 8 consumer warps, 2 CTAs/SM; 1: 6 x 16 KiB, 2: 5 x 16 KiB,
  * 3: 4 x 16 KiB; 4: 6 x 32 KiB, 16 consumer warps, 1 CTA/SM; 5: 5 x 32 KiB, 16 warps;
  * 6: 4 x 32 KiB, 16 warps; 7: 3 x 16 KiB, 4 consumer warps, 4 CTAs/SM; 8: 4 x 16 KiB,
- * 4 warps, 3 CTAs/SM; -1 = default / the CSWAP_ZVC_CFG environment variable).
- * Process-wide; returns CSWAP_ERR_INVALID for a variant outside -1..8. */
+ * 4 warps, 3 CTAs/SM; 9: 4 x 24 KiB, 8 consumer warps, 2 CTAs/SM; -1 = default / the
+ * CSWAP_ZVC_CFG environment variable).
+ * Process-wide; returns CSWAP_ERR_INVALID for a variant outside -1..9. */
 cswap_status cswap_set_zvc_launch(uint32_t grid, int32_t variant);
 
 /* ---- device codecs (a3-a10) ------------------------------------------------------------------ */

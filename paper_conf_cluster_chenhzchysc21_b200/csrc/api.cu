@@ -1100,7 +1100,7 @@ cswap_status cswap_set_format(const cswap_format* f) {
 }
 
 cswap_status cswap_set_zvc_launch(uint32_t grid, int32_t variant) {
-  if (!zvc_set_launch(grid, variant)) return fail(CSWAP_ERR_INVALID, "variant %d outside -1..8", int(variant));
+  if (!zvc_set_launch(grid, variant)) return fail(CSWAP_ERR_INVALID, "variant %d outside -1..9", int(variant));
   return CSWAP_OK;
 }
 

@@ -959,7 +959,7 @@ static cudaError_t launch_compress_s(const void* in, uint64_t n, uint64_t F, uin
 }
 
 // compress configuration (stages x tile bytes): cswap_set_zvc_launch, else CSWAP_ZVC_CFG, else 0
-constexpr int kMaxVariant = 8;
+constexpr int kMaxVariant = 9;
 static int compress_cfg() {
   const int v = g_zvc_variant.load(std::memory_order_relaxed);
   if (v >= 0) return v;
@@ -995,6 +995,9 @@ static cudaError_t launch_compress_t(const void* in, uint64_t n, uint64_t F, uin
     // (barriers, the offset wait) of 3-4 resident tiles overlap
     case 7: return launch_compress_s<T, 3, 4, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
     case 8: return launch_compress_s<T, 4, 4, 16384>(in, n, F, out, out_size, sc, epoch, dtype, st);
+    // the same 96 KiB of stages as 4 x 24 KiB: LAG = 2 tile periods for the offset to resolve
+    // (the default's consumers wait ~1000-1300 cycles per tile for it, CSWAP_ZVC_PROF)
+    case 9: return launch_compress_s<T, 4, 8, 24576>(in, n, F, out, out_size, sc, epoch, dtype, st);
     default: return launch_compress_s<T, 3, 8, 32768>(in, n, F, out, out_size, sc, epoch, dtype, st);
   }
 }

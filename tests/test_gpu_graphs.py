@@ -92,22 +92,24 @@ def test_plain_launch_path_matches():
 
 
 @pytest.mark.parametrize("grid,variant", [(1, 0), (7, 1), (148, 2), (296, 3), (0, 4), (5, 5),
-                                           (148, 6), (0, 7), (300, 8), (0, -1)])
-def test_zvc_launch_config_keeps_bytes(C, grid, variant):
-    """cswap_set_zvc_launch changes only how the persistent compress runs, never its bytes."""
-    n = (1 << 21) + 333
-    x = synth.relu_iid(n, 0.45, seed=11)
-    ref = O.compress(x, O.ZVC, O.F32)
+                                           (148, 6), (0, 7), (300, 8), (0, 9), (3, 9), (0, -1)])
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_zvc_launch_config_keeps_bytes(C, grid, variant, dtype):
+    """cswap_set_zvc_launch changes only how the persistent compress runs, never its bytes (incl.
+    variant 9's 24 KiB tiles: 683 tiles per 2^22-element frame, a short last tile per frame)."""
+    n = (9 << 20) + 333 if dtype == 0 else (17 << 20) + 77  # 3 / 5 frames, ragged
+    x = synth.relu_iid(n, 0.45, seed=11, dtype=dtype)
+    ref = O.compress(x, O.ZVC, dtype)
     try:
         C.set_zvc_launch(grid, variant)
-        assert G.gpu_compress(C, x, O.ZVC, O.F32) == ref
+        assert G.gpu_compress(C, x, O.ZVC, dtype) == ref
     finally:
         C.set_zvc_launch(0, -1)
 
 
 def test_zvc_launch_config_rejects_bad_variant(C):
     with pytest.raises(C.CswapError):
-        C.set_zvc_launch(0, 9)
+        C.set_zvc_launch(0, 10)
 
 
 def test_timing_records_carry_device_clock(C):
