@@ -60,11 +60,17 @@ class ClockSampler:
         self.proc = None
 
     def __enter__(self):
+        self.first = ""
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.device), "--query-gpu=" + ",".join(self.FIELDS),
                  "--format=csv,noheader,nounits", "-lms", "200"], stdout=subprocess.PIPE,
                 stderr=subprocess.DEVNULL, text=True)
+            # wait for the first sample: nvidia-smi's start-up (NVML init, first query) then falls
+            # before the caller's warm-up and timed steps, not inside them
+            import select
+            if select.select([self.proc.stdout], [], [], 10.0)[0]:
+                self.first = self.proc.stdout.readline()
         except OSError:
             self.proc = None
         return self
@@ -77,6 +83,7 @@ class ClockSampler:
                 self.out, _ = self.proc.communicate(timeout=5)
             except subprocess.TimeoutExpired:
                 self.proc.kill()
+        self.out = getattr(self, "first", "") + (self.out or "")
 
     def summary(self) -> dict:
         sms, mx, reasons = [], None, set()
@@ -160,7 +167,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
     def timed(codec, steps, warmup, record=False, clocks=False):
         # the clock sampler starts before the warm-up so that nvidia-smi is already sampling
         # (every 200 ms) when the short timed region begins; it stops right after it
-        sampler = ClockSampler(local_rank) if clocks else None
+        sampler = ClockSampler(local_rank) if clocks and not os.environ.get("BENCH_NO_CLOCKS") else None
         if sampler:
             sampler.__enter__()
         for _ in range(warmup):

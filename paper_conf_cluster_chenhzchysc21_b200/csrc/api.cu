@@ -718,6 +718,7 @@ cswap_status check_common(const void* p, const char* what) {
 struct cswap_handle {
   Ctx* ctx = nullptr;
   uint8_t* host = nullptr;  // container (pinned pool): allocated at the codec's worst case, trimmed
+  uint8_t* host_base = nullptr;  // the pool allocation `host` lies in (host = host_base + alignment pad)
   uint64_t bytes = 0;       // container bytes (valid once out_state != 0)
   uint64_t cap = 0;         // bytes allocated at `host`
   uint64_t n = 0;
@@ -756,7 +757,25 @@ struct OutJob {
   cudaEvent_t done;  // recorded on the caller's stream after the compress group
   bool exact_host;   // frames arrive all at once: allocate the host container at its exact size
   uint64_t cap;      // staging bytes (the codec's worst case)
+  uint8_t* staging_base;  // the pool allocation (staging = staging_base + alignment pad)
 };
+
+// DMA alignment: a D2H copy whose host destination is not 64-byte aligned runs at 52.3 GB/s,
+// an aligned one at 57.1 (tools/d2h_step_probe.py: the same 784 MiB copy into the library's pinned
+// container at its 80-byte data offset vs into a torch pinned tensor).  Containers are therefore
+// placed in their pinned allocation so that `h->host` has a chosen residue mod 256 (the staging
+// buffer's, or the raw tensor's minus the data offset), and copies start at 256-aligned addresses.
+constexpr uintptr_t kDmaAlign = 256;
+bool alloc_host(Ctx* c, cswap_handle* h, uint64_t bytes, uintptr_t residue) {
+  h->host_base = c->pinned.alloc(bytes + kDmaAlign);
+  if (!h->host_base) {
+    h->host = nullptr;
+    return false;
+  }
+  h->host = h->host_base + ((residue - reinterpret_cast<uintptr_t>(h->host_base)) & (kDmaAlign - 1));
+  return true;
+}
+inline uintptr_t addr(const void* p) { return reinterpret_cast<uintptr_t>(p); }
 
 void finish_out(cswap_handle* h, int state, cswap_status err, const std::string& msg) {
   {
@@ -854,7 +873,7 @@ void run_out_job(Ctx* c, OutJob* j) {
     if (j->exact_host && k_ready == j->K && !h->host) {
       // every frame is published at once (publication after the codec's last kernel): pin the
       // container at its exact size (no worst-case allocation: RLE / CSR reserve 2-3x raw)
-      h->host = c->pinned.alloc(h->ends.back());
+      alloc_host(c, h, h->ends.back(), addr(j->staging));  // host == staging (mod 256)
       h->cap = h->ends.back();
       if (!h->host) {
         err = CSWAP_ERR_NOMEM;
@@ -873,8 +892,13 @@ void run_out_job(Ctx* c, OutJob* j) {
         std::this_thread::yield();
         continue;
       }
+      // start at the 256-aligned address at or below pos (re-copying up to 255 bytes the previous
+      // copy already moved: the staging bytes are final), never below the data start
+      uint64_t start = pos;
+      if (pos > ds) start = std::max<uint64_t>(ds, pos - (addr(j->staging + pos) & (kDmaAlign - 1)));
       if (end > pos &&
-          cudaMemcpyAsync(h->host + pos, j->staging + pos, end - pos, cudaMemcpyDeviceToHost, c->s_d2h) != cudaSuccess) {
+          cudaMemcpyAsync(h->host + start, j->staging + start, end - start, cudaMemcpyDeviceToHost, c->s_d2h) !=
+              cudaSuccess) {
         err = CSWAP_ERR_CUDA;
         msg = cudaGetErrorString(cudaGetLastError());
         break;
@@ -905,7 +929,7 @@ void run_out_job(Ctx* c, OutJob* j) {
     else std::this_thread::sleep_for(std::chrono::microseconds(20));
   }
   if (err == CSWAP_OK && !h->host) {  // n = 0: a header-only container
-    h->host = c->pinned.alloc(pos);
+    alloc_host(c, h, pos, 0);
     h->cap = pos;
     if (!h->host) {
       err = CSWAP_ERR_NOMEM;
@@ -916,13 +940,13 @@ void run_out_job(Ctx* c, OutJob* j) {
   // staging is freed on the D2H stream behind the copies; when nothing waited for the kernels
   // (a failure, or n = 0 with no frame to publish) the free is ordered behind the group itself
   if (err != CSWAP_OK || j->K == 0) cudaStreamWaitEvent(c->s_d2h, j->done, 0);
-  cudaFreeAsync(j->staging, c->s_d2h);
+  cudaFreeAsync(j->staging_base, c->s_d2h);
   cudaEventRecord(h->ev_out, c->s_d2h);
   cudaEventDestroy(j->done);
   c->small.free(reinterpret_cast<uint8_t*>(j->prog));  // the kernel has written its last word
   if (err == CSWAP_OK) {
     h->bytes = pos;
-    c->pinned.shrink(h->host, pos);
+    c->pinned.shrink(h->host_base, uint64_t(h->host - h->host_base) + pos);
     h->cap = pos;
   }
   finish_out(h, err == CSWAP_OK ? 1 : 2, err, msg);
@@ -1416,7 +1440,7 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     // raw offload (vDNN): the host writes header + frame table, the copy engine
     // moves the tensor's bytes straight into the frames after the caller's stream reaches here
     const uint64_t cap = max_size(n, w, CSWAP_CODEC_NONE, f);
-    h->host = c->pinned.alloc(cap);
+    alloc_host(c, h, cap, addr(d_in) - ds);  // host + ds == d_in (mod 256): aligned raw copies
     if (!h->host) return bail(fail(CSWAP_ERR_NOMEM, "pinned alloc of %llu B failed", (unsigned long long)cap));
     h->cap = cap;
     const uint64_t tail = ds + uint64_t(w) * n;
@@ -1447,9 +1471,12 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
   // finished frame; the executor thread copies frames to the pinned host container as they are
   // published.  Nothing here waits for the device.
   const uint64_t cap = max_size(n, w, use, f);
-  uint8_t* staging = nullptr;
-  if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging), cap, c->pool, st) != cudaSuccess)
+  // staging placed so that its data start (staging + ds) is 256-aligned: the first copy of every
+  // container starts aligned, later copies start at aligned addresses at or below their frame
+  uint8_t* staging_base = nullptr;
+  if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging_base), cap + kDmaAlign, c->pool, st) != cudaSuccess)
     return bail(fail(CSWAP_ERR_NOMEM, "device staging of %llu B failed", (unsigned long long)cap));
+  uint8_t* staging = staging_base + ((uintptr_t(0) - ds - addr(staging_base)) & (kDmaAlign - 1));
   // per-frame publication pays only when the D2H link would otherwise wait for this tensor's
   // compression (nothing queued ahead of it); CSWAP_FRAME_PUBLISH=0/1 forces it off/on.  Only
   // ZVC publishes from inside its kernel; then the host container is pinned at the worst case
@@ -1463,12 +1490,12 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
   }
   frame_publish = frame_publish && use == CSWAP_CODEC_ZVC;
   if (frame_publish) {
-    h->host = c->pinned.alloc(cap);
+    alloc_host(c, h, cap, addr(staging));  // host == staging (mod 256)
     h->cap = cap;
   }
   uint64_t* prog = reinterpret_cast<uint64_t*>(c->small.alloc(8ull * std::max<uint32_t>(K, 1)));
   if ((frame_publish && !h->host) || !prog) {
-    cudaFreeAsync(staging, st);
+    cudaFreeAsync(staging_base, st);
     c->small.free(reinterpret_cast<uint8_t*>(prog));
     return bail(fail(CSWAP_ERR_NOMEM, "pinned alloc of %llu B failed", (unsigned long long)cap));
   }
@@ -1488,12 +1515,12 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     s = fail(CSWAP_ERR_CUDA, "event record failed");
   if (s != CSWAP_OK) {
     if (done) cudaEventDestroy(done);
-    cudaFreeAsync(staging, st);
+    cudaFreeAsync(staging_base, st);
     cudaStreamSynchronize(st);  // the group may have been partly enqueued: prog is still referenced
     c->small.free(reinterpret_cast<uint8_t*>(prog));
     return bail(s);
   }
-  enqueue_out(c, new OutJob{h, staging, prog, K, done, !frame_publish, cap});
+  enqueue_out(c, new OutJob{h, staging, prog, K, done, !frame_publish, cap, staging_base});
   *out = h;
   return CSWAP_OK;
 }
@@ -1537,9 +1564,13 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
   // pipelined prefetch per frame (R7; the pipelined cost model's K): frame k's H2D overlaps the
   // decompression of frame k-1.  Staging is allocated on the first copy stream, which the
   // second copy stream follows; consecutive frames alternate between the two copy streams.
-  uint8_t* staging = nullptr;
-  if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging), h->bytes, c->pool, c->s_h2d) != cudaSuccess)
+  // staging == host (mod 256), and every H2D step starts at a 256-aligned address at or below
+  // its first byte (re-reading up to 255 bytes of the previous step: identical values)
+  uint8_t* staging_base = nullptr;
+  if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging_base), h->bytes + kDmaAlign, c->pool, c->s_h2d) !=
+      cudaSuccess)
     return fail(CSWAP_ERR_NOMEM, "swap-in staging of %llu B failed", (unsigned long long)h->bytes);
+  uint8_t* staging = staging_base + ((addr(h->host) - addr(staging_base)) & (kDmaAlign - 1));
   std::vector<cudaEvent_t> evs;
   cswap_status s = CSWAP_OK;
   cudaEvent_t alloc_ev;
@@ -1581,7 +1612,8 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
         break;
       }
       evs.push_back(e);
-      if (cudaMemcpyAsync(staging + off, h->host + off, end - off, cudaMemcpyHostToDevice, cs) != cudaSuccess ||
+      const uint64_t start = off - (off ? (addr(h->host + off) & (kDmaAlign - 1)) : 0);
+      if (cudaMemcpyAsync(staging + start, h->host + start, end - start, cudaMemcpyHostToDevice, cs) != cudaSuccess ||
           cudaEventRecord(e, cs) != cudaSuccess || cudaStreamWaitEvent(st, e, 0) != cudaSuccess) {
         s = fail(CSWAP_ERR_CUDA, "prefetch copy failed");
         break;
@@ -1613,7 +1645,7 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
     }
   }
   // every staging read is on st (the last decode); frees and the end event follow it there
-  cudaFreeAsync(staging, st);
+  cudaFreeAsync(staging_base, st);
   cudaEventRecord(h->ev_in, st);
   for (auto e : evs) cudaEventDestroy(e);
   return s;
@@ -1663,7 +1695,7 @@ void cswap_handle_free(cswap_handle* h) {
   if (h->ev_out) cudaEventDestroy(h->ev_out);
   if (h->ev_in) cudaEventDestroy(h->ev_in);
   if (h->dev) cudaFreeAsync(h->dev, h->ctx->s_d2h);  // every use is complete (events above)
-  h->ctx->pinned.free(h->host);
+  h->ctx->pinned.free(h->host_base);
   h->ctx->small.free(h->slots);
   delete h;
 }
