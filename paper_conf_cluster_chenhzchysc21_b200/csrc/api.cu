@@ -883,9 +883,8 @@ void run_out_job(Ctx* c, OutJob* j) {
     }
     if (k_ready > k && (!j->exact_host || k_ready == j->K)) {  // exact_host: the whole container at once
       const uint64_t end = h->ends[k_ready - 1];
-      // copy granularity: a D2H copy costs a few us of DMA ramp and tail (8 MiB copies ran at
-      // 52.2 GB/s, whole tensors at 54.0, tools/pipeline_probe.py), so published frames are
-      // coalesced until `min_copy` bytes are ready -- unless the D2H stream is idle (then any
+      // copy granularity: every D2H copy costs a few us of DMA ramp and tail, so published frames
+      // are coalesced until `min_copy` bytes are ready -- unless the D2H stream is idle (then any
       // frame goes at once: this is what overlaps a tensor's first frames with its compression)
       // or every frame is published
       if (k_ready < j->K && end - pos < min_copy && cudaStreamQuery(c->s_d2h) == cudaErrorNotReady) {
@@ -894,8 +893,7 @@ void run_out_job(Ctx* c, OutJob* j) {
       }
       // start at the 256-aligned address at or below pos (re-copying up to 255 bytes the previous
       // copy already moved: the staging bytes are final), never below the data start
-      uint64_t start = pos;
-      if (pos > ds) start = std::max<uint64_t>(ds, pos - (addr(j->staging + pos) & (kDmaAlign - 1)));
+      const uint64_t start = pos - std::min<uint64_t>(pos - ds, addr(j->staging + pos) & (kDmaAlign - 1));
       if (end > pos &&
           cudaMemcpyAsync(h->host + start, j->staging + start, end - start, cudaMemcpyDeviceToHost, c->s_d2h) !=
               cudaSuccess) {
@@ -940,6 +938,7 @@ void run_out_job(Ctx* c, OutJob* j) {
   // staging is freed on the D2H stream behind the copies; when nothing waited for the kernels
   // (a failure, or n = 0 with no frame to publish) the free is ordered behind the group itself
   if (err != CSWAP_OK || j->K == 0) cudaStreamWaitEvent(c->s_d2h, j->done, 0);
+  if (err != CSWAP_OK) cudaEventSynchronize(j->done);  // the kernels may still write progress words
   cudaFreeAsync(j->staging_base, c->s_d2h);
   cudaEventRecord(h->ev_out, c->s_d2h);
   cudaEventDestroy(j->done);
@@ -1612,7 +1611,7 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
         break;
       }
       evs.push_back(e);
-      const uint64_t start = off - (off ? (addr(h->host + off) & (kDmaAlign - 1)) : 0);
+      const uint64_t start = off - std::min<uint64_t>(off, addr(h->host + off) & (kDmaAlign - 1));
       if (cudaMemcpyAsync(staging + start, h->host + start, end - start, cudaMemcpyHostToDevice, cs) != cudaSuccess ||
           cudaEventRecord(e, cs) != cudaSuccess || cudaStreamWaitEvent(st, e, 0) != cudaSuccess) {
         s = fail(CSWAP_ERR_CUDA, "prefetch copy failed");
