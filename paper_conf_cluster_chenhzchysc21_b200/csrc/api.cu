@@ -1560,9 +1560,9 @@ cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream) {
     return s;
   }
   CU(cudaStreamWaitEvent(c->s_h2d2, h->ev_out, 0));
-  // pipelined prefetch per frame (R7; the pipelined cost model's K): frame k's H2D overlaps the
-  // decompression of frame k-1.  Staging is allocated on the first copy stream, which the
-  // second copy stream follows; consecutive frames alternate between the two copy streams.
+  // pipelined prefetch in groups of whole frames (R7, R22; the cost model's G): group g's H2D
+  // overlaps the decompression of group g-1.  Staging is allocated on the first copy stream,
+  // which the second copy stream follows; consecutive groups alternate between the two streams.
   // staging == host (mod 256), and every H2D step starts at a 256-aligned address at or below
   // its first byte (re-reading up to 255 bytes of the previous step: identical values)
   uint8_t* staging_base = nullptr;

@@ -54,8 +54,8 @@ for task in "$@"; do
   profiles)
     timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/p_launches.csv python bench.py --steps 2 --warmup 3 --no-extras --no-cpu > gpurun_out/p_launches.log 2>&1
     python tools/launch_summary.py gpurun_out/p_launches.csv "python bench.py --steps 2 --warmup 3 --no-extras --no-cpu (under ncu: warm-up + timed steps of the VGG16 b64 set, then the isolated replay of the 12 tensors x 4)" > gpurun_out/p_launches.txt
-    timeout 1200 ncu --set full --clock-control none -k regex:zvc_compress -s 36 -c 12 -o $R/bench_step -f python bench.py --steps 1 --warmup 3 --no-extras --no-cpu > gpurun_out/p_ncu1.log 2>&1
-    timeout 1200 ncu --set full --clock-control none -k regex:"zvc_(count|scan|expand)" -s 120 -c 30 -o $R/bench_dec -f python bench.py --steps 1 --warmup 3 --no-extras --no-cpu > gpurun_out/p_ncu2.log 2>&1
+    timeout 1200 ncu --set full --clock-control none -k regex:zvc_compress -s 37 -c 12 -o $R/bench_step -f python bench.py --steps 1 --warmup 3 --no-extras --no-cpu > gpurun_out/p_ncu1.log 2>&1
+    timeout 1200 ncu --set full --clock-control none -k regex:"zvc_(count|scan|expand)" -s 369 -c 30 -o $R/bench_dec -f python bench.py --steps 1 --warmup 3 --no-extras --no-cpu > gpurun_out/p_ncu2.log 2>&1
     for d in f32 f16; do
       timeout 600 ncu --set full --import-source on --clock-control none -k regex:"zvc_(compress_persistent|expand)" -s 2 -c 2 -o $R/micro_$d -f python tools/codec_bench.py --codecs zvc --mib 1024 --s 0.5 --dtype $d --ncu > gpurun_out/p_ncu_micro_$d.log 2>&1
       python tools/ncu_sass_mix.py $R/micro_$d.ncu-rep zvc_compress 25 > gpurun_out/p_sassmix_compress_$d.txt 2>&1
