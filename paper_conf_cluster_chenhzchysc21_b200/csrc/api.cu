@@ -582,9 +582,10 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
     c->launches++;
     return cuda_status(launch_publish_frames(out, K, prog, gs), "publish_frames");
   };
-  auto with_prog = [&](const Scratch& sc) {
+  auto with_prog = [&](const Scratch& sc, uint32_t mode) {
     Scratch s2 = sc;
     s2.prog = prog;
+    s2.prog_mode = prog ? mode : 0;
     return s2;
   };
   if (n == 0) {
@@ -606,14 +607,17 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       // per-frame publication from inside the persistent kernel only when asked (the D2H link
       // is idle, so the first frames' copies can overlap the rest of the compression); it costs
       // the kernel ~14 us (a gpu-scope acq_rel atomic per tile in the producer warp), so a
-      // swap-out queued behind other copies publishes after the kernel instead
-      const bool inkernel = prog && frame_publish;
-      return run_group(c, st, group_key(kGrpCompress, codec, dtype) | (inkernel ? 1u << 21 : 0u), [&](cudaStream_t gs) {
-        TRY(cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, inkernel ? with_prog(L.b->sc) : L.b->sc, ep,
-                                            dtype, gs),
-                        "zvc_compress"));
-        return inkernel ? CSWAP_OK : publish(gs);
-      });
+      // swap-out queued behind other copies has the kernel's last CTA publish every frame at
+      // the end instead (no extra launch)
+      static const bool end_kernel = getenv("CSWAP_ZVC_ENDPUB") && getenv("CSWAP_ZVC_ENDPUB")[0] == '0';  // A/B
+      const uint32_t mode = frame_publish ? 1 : (end_kernel ? 0 : 2);
+      return run_group(c, st, group_key(kGrpCompress, codec, dtype) | (mode == 0 && prog ? 1u << 21 : 0u),
+                       [&](cudaStream_t gs) {
+                         TRY(cuda_status(launch_zvc_compress(in, n, w, F, out, out_size,
+                                                             mode ? with_prog(L.b->sc, mode) : L.b->sc, ep, dtype, gs),
+                                         "zvc_compress"));
+                         return mode == 0 ? publish(gs) : CSWAP_OK;
+                       });
     }
     case CSWAP_CODEC_RLE: {
       Lease L(*c, st, rle_tiles(n, w, F) + 2, uint64_t(K) + 2);

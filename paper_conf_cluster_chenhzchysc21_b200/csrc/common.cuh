@@ -44,6 +44,9 @@ struct Scratch {
   // group stores kProgReady | (end offset of frame k in the container) once every byte of frame
   // k (and its frame-table entry) is in device memory, so the host can start that frame's D2H
   uint64_t* prog;
+  // ZVC compress only: 1 = publish each frame as soon as it is complete (the producer warps),
+  // 2 = the last CTA publishes every frame once the kernel is done (no extra launch)
+  uint32_t prog_mode;
 };
 constexpr uint64_t kProgReady = 1ull << 63;
 

@@ -233,7 +233,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     // both written before the frame's last tiles were emitted) for the host's per-frame D2H
     uint64_t* const fdone = sc.zacc + K + uint64_t(K) * gpf;  // after the accumulators
     auto tile_emitted = [&](uint32_t t) {
-      if (!sc.prog || lane != 0) return;
+      if (!sc.prog || sc.prog_mode != 1 || lane != 0) return;
       uint32_t k, j, te, be;
       uint64_t Fk;
       tile_geom(t, k, j, Fk, te, be);
@@ -273,7 +273,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         }
         if (done_t != SENT) tile_emitted(done_t);
         // the tiles of rounds i-S+1 .. i-1 are still being emitted: wait for each and count it
-        if (sc.prog) {
+        if (sc.prog && sc.prog_mode == 1) {
           for (uint32_t p = i >= uint32_t(S - 1) ? i - (S - 1) : 0; p < i; p++) {
             producer_wait(&bar_empty[p % S], (p / S) & 1);
             if (lane == 0) tile_emitted(s_ticket[p % S]);
@@ -600,6 +600,13 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
   if (s_last) {
     for (uint64_t q = tid; q < nacc; q += blockDim.x) sc.zacc[q] = 0;
     if (tid == 0) sc.zacc[nacc] = 0;
+    // swap-out progress published at the end (prog_mode 2): every tile of every CTA is emitted
+    // (each CTA's done-count release covers its stores; this CTA acquired all of them), so the
+    // frame starts and frame-table entries are final
+    if (sc.prog && sc.prog_mode == 2)
+      for (uint32_t k = tid; k < K; k += blockDim.x)
+        publish_frame(sc.prog, k, status_value(ld_relaxed(sc.aux + k)) +
+                                      ld_relaxed(reinterpret_cast<const uint64_t*>(out + 64) + k));
   }
 }
 
