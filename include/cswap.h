@@ -160,20 +160,32 @@ cswap_status cswap_select(const void* d_in, uint64_t n, cswap_dtype dtype, doubl
                           void* stream, cswap_decision* out);
 
 /* ---- swap pipeline (a11, a12) --------------------------------------------------------------- */
-/* Swap d_in out to library-owned pinned host memory, compressed with `codec` (AUTO: probe +
- * selector with the given hidden times, PAPER.md:139 Hidden_f/Hidden_b).  Work is ordered after
- * everything already queued on `stream`.  d_in must stay unmodified until cswap_handle_wait()
- * returns or cswap_handle_record_out() 's event is waited on. */
+/* Swap d_in out to library-owned pinned host memory (or the cswap_set_swap_target device),
+ * compressed with `codec` (AUTO: probe + selector with the given hidden times, PAPER.md:139
+ * Hidden_f/Hidden_b).  Work is ordered after everything already queued on `stream`.
+ * Asynchronous: with a fixed codec the call only enqueues the codec kernels on `stream` and hands
+ * the copies to the library's executor thread (frames are copied D2H as the kernels publish
+ * them) -- it never waits for the device.  AUTO first waits
+ * for the probe's counts (the selector runs on the host).
+ * Lifetime of d_in: for a compressing codec d_in is read only by kernels on `stream`, so work
+ * queued on `stream` afterwards may overwrite it; for CSWAP_CODEC_NONE (raw copy on the library's
+ * copy stream) d_in must stay unmodified until cswap_handle_wait() returns or a stream has waited
+ * through cswap_handle_record_out(). */
 cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, cswap_codec codec, double hidden_f,
                             double hidden_b, void* stream, cswap_handle** out);
 /* Restore the tensor into d_out (n elements, device), ordered on `stream`: kernels queued on
- * `stream` afterwards see the restored data.  The handle keeps its host copy (swap-in may be
- * repeated) until cswap_handle_free. */
+ * `stream` afterwards see the restored data.  Waits (on the host) only until the swap-out's
+ * copies have been issued; the H2D copies are ordered after the D2H on the device.  The handle
+ * keeps its host copy (swap-in may be repeated) until cswap_handle_free. */
 cswap_status cswap_swap_in(cswap_handle* h, void* d_out, void* stream);
-/* Block until every swap operation on h finished; returns deferred asynchronous errors. */
+/* Block until every swap operation on h finished (D2H, and H2D + decode if swap-in was issued);
+ * returns deferred asynchronous errors (CORRUPT for a container that failed validation). */
 cswap_status cswap_handle_wait(cswap_handle* h);
 /* Make `stream` wait (device-side) until h's swap-out finished (d_in reusable). */
 cswap_status cswap_handle_record_out(cswap_handle* h, void* stream);
+/* codec and decision are known when cswap_swap_out returns (pass NULL for the rest to avoid any
+ * wait); container_bytes / host_container wait until the swap-out's copies are issued (the host
+ * bytes are complete once cswap_handle_wait returns).  host_container is NULL for a device target. */
 cswap_status cswap_handle_query(const cswap_handle* h, cswap_codec* codec, uint64_t* container_bytes,
                                 const void** host_container, cswap_decision* decision);
 void cswap_handle_free(cswap_handle* h);
