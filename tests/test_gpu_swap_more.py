@@ -151,3 +151,26 @@ def test_bert_like_fp16_set_selection(C):
         torch.cuda.synchronize()
         assert np.array_equal(G.from_dev(out)[:n], x)
         h.close()
+
+
+def test_bench_two_ranks_on_one_gpu():
+    """bench.py --gpus 2 end to end on the GPU box (both ranks share GPU 0 via BENCH_SHARE_GPU,
+    so this checks the launcher / gloo barrier / max-over-ranks / gather path with the real swap
+    workload, not scaling): one JSON line, n_gpus = 2, per-rank entries, value = 2 x raw / max."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = {k: v for k, v in os.environ.items() if k not in ("RANK", "LOCAL_RANK", "WORLD_SIZE", "MASTER_ADDR",
+                                                            "MASTER_PORT")}
+    env["BENCH_SHARE_GPU"] = "1"
+    p = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--steps", "2", "--warmup", "3",
+                        "--no-extras", "--no-cpu"], capture_output=True, text=True, timeout=900, env=env, cwd=root)
+    assert p.returncode == 0, p.stderr[-3000:]
+    lines = [ln for ln in p.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    res = json.loads(lines[0])
+    assert res["n_gpus"] == 2 and len(res["per_rank"]) == 2
+    raw = res["config"]["raw_MiB_per_gpu"] * 2**20
+    assert abs(res["value"] - 2 * raw / (res["ms_per_step"] * 1e-3) / 1e9) < 0.01 * res["value"]
