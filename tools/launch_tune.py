@@ -3,8 +3,8 @@ Alg. 1, :170-214; Fig. 5 and Fig. 12 analogues).
 
 Objective: Time_c + Time_dc of one synthetic 500 MB tensor at 50 % sparsity.
 The B200 knob: the persistent compress kernel's grid q (1 .. co-resident maximum, SMs x 2) and
-its stage/tile variant v (0..3, which also sets the block size: 384/480/448/416 threads) —
-cswap_set_zvc_launch.  The decode kernels take one CTA per tile (no free grid parameter).
+its stage/tile variant v (0..9: stages x tile bytes x consumer warps, see cswap.h, which also sets
+the block size and the resident CTAs per SM) — cswap_set_zvc_launch.  The decode kernels take one CTA per tile (no free grid parameter).
 
 Searches compared (Fig. 12): Alg. 1 Bayesian optimisation (s1 = 10 random
 points, then s2 = 25 points chosen by expected improvement under a Gaussian-process posterior,
@@ -12,7 +12,7 @@ written out below with numpy — the paper used fmfn/BayesianOptimization [47], 
 here), random search with the same 35 evaluations, the "expert" default (q = SMs x 2, v = 0) and
 the exhaustive grid (every q x v: Fig. 5's full curve).
 
-    python tools/launch_tune.py [--mb 500] [--s 0.5] [--reps 5] [--out profiles/launch_tune_r01.json]
+    python tools/launch_tune.py [--mb 500] [--s 0.5] [--reps 5] [--out profiles/launch_tune_r02.json]
 """
 import argparse
 import json
@@ -137,7 +137,8 @@ def main():
         return sorted(ts)[len(ts) // 2]
 
     grids = list(range(1, 2 * sms + 1))
-    space = [(q, v) for v in range(4) for q in grids]
+    NV = 10
+    space = [(q, v) for v in range(NV) for q in grids]
     res = {"objective": f"Time_c + Time_dc (ms), ZVC, {a.mb:.0f} MB fp32 at s = {a.s}", "sms": sms}
     t0 = time.time()
     expert = evaluate((0, 0))
@@ -158,7 +159,7 @@ def main():
     gp_, gy = min(full.items(), key=lambda t: t[1])
     res["grid_search"] = {"best": {"q": gp_[0], "v": gp_[1], "ms": round(gy, 4)}, "evaluations": len(space),
                           "seconds": round(time.time() - t0, 2)}
-    res["fig5_curve_ms"] = {f"v{v}": [round(full[(q, v)], 4) for q in grids] for v in range(4)}
+    res["fig5_curve_ms"] = {f"v{v}": [round(full[(q, v)], 4) for q in grids] for v in range(NV)}
     C.set_zvc_launch(0, -1)
     print(json.dumps({k: v for k, v in res.items() if k != "fig5_curve_ms"}, indent=1))
     with open(a.out, "w") as f:
