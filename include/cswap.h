@@ -208,6 +208,12 @@ cswap_status cswap_get_swap_target(int* device);
  * before returning.  Works for every target. */
 cswap_status cswap_handle_copy_container(cswap_handle* h, void* dst, uint64_t cap, void* stream);
 
+/* Give cached memory back (like torch.cuda.empty_cache): trims the library's device staging pool
+ * to `keep_bytes` (cudaMemPoolTrimTo; the pool otherwise keeps up to CSWAP_POOL_KEEP_MB, default
+ * 16 GiB, so that steady swapping never re-maps memory) and unpins host chunks that hold no live
+ * container.  Synchronises the device first. */
+cswap_status cswap_release_cached(uint64_t keep_bytes);
+
 /* ---- calibration (a13) ----------------------------------------------------------------------- */
 /* Ordinary least squares t = b0 + b1*S + b2*S*s over m samples ("linear
  * regression"); beta_out[3].  Returns CSWAP_ERR_INVALID if m < 3 or the design is singular. */

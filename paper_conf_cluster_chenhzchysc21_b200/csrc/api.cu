@@ -159,6 +159,27 @@ struct PinnedPool {
     chunks.clear();
     live.clear();
   }
+  // unpin chunks that hold no live allocation (indices in `live` are renumbered)
+  uint64_t release_empty() {
+    std::lock_guard<std::mutex> lk(m);
+    std::vector<bool> used(chunks.size(), false);
+    for (auto& kv : live) used[kv.second.first] = true;
+    std::vector<size_t> remap(chunks.size(), SIZE_MAX);
+    std::vector<Chunk> keep;
+    uint64_t freed = 0;
+    for (size_t c = 0; c < chunks.size(); c++) {
+      if (used[c]) {
+        remap[c] = keep.size();
+        keep.push_back(std::move(chunks[c]));
+      } else {
+        cudaFreeHost(chunks[c].base);
+        freed += chunks[c].size;
+      }
+    }
+    for (auto& kv : live) kv.second.first = remap[kv.second.first];
+    chunks = std::move(keep);
+    return freed;
+  }
 };
 
 // ---------------------------------------------------------------------------------------------
@@ -1712,6 +1733,17 @@ cswap_status cswap_handle_copy_container(cswap_handle* h, void* dst, uint64_t ca
   CU(cudaStreamWaitEvent(st, h->ev_out, 0));
   CU(cudaMemcpyAsync(dst, h->dev ? static_cast<const void*>(h->dev) : h->host, bytes, cudaMemcpyDefault, st));
   CU(cudaStreamSynchronize(st));
+  return CSWAP_OK;
+}
+
+cswap_status cswap_release_cached(uint64_t keep_bytes) {
+  Ctx* c = nullptr;
+  TRY(need_ctx(&c));
+  CU(cudaDeviceSynchronize());
+  CU(cudaMemPoolTrimTo(c->pool, keep_bytes));
+  if (c->tpool) CU(cudaMemPoolTrimTo(c->tpool, keep_bytes));
+  c->pinned.release_empty();
+  c->small.release_empty();
   return CSWAP_OK;
 }
 

@@ -112,6 +112,7 @@ _SIGS = {
     "cswap_set_swap_target": (_i, [_i]),
     "cswap_get_swap_target": (_i, [_P(ctypes.c_int)]),
     "cswap_handle_copy_container": (_i, [_vp, _vp, _u64, _vp]),
+    "cswap_release_cached": (_i, [_u64]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_L, _name)
@@ -294,6 +295,11 @@ class Handle:
 def set_swap_target(device: int = -1):
     """-1 = pinned host memory (default); else a device (this one or a peer over NVLink)."""
     _check(_L.cswap_set_swap_target(device), "cswap_set_swap_target")
+
+
+def release_cached(keep_bytes: int = 0):
+    """Trim the staging pool to keep_bytes and unpin empty host chunks (like torch.cuda.empty_cache)."""
+    _check(_L.cswap_release_cached(keep_bytes), "cswap_release_cached")
 
 
 def get_swap_target() -> int:

@@ -138,3 +138,26 @@ def test_corrupted_multiframe_host_container_is_reported(C, codec):
         torch.cuda.synchronize()
     finally:
         C.set_format(1 << 22, 1024, 65536)
+
+
+def test_release_cached_keeps_live_containers(C):
+    """cswap_release_cached trims the staging pool and unpins empty host chunks; live containers
+    stay intact and restorable."""
+    n = 3 << 20
+    x = synth.relu_iid(n, 0.5, seed=404)
+    d = G.to_dev(x)
+    live = C.swap_out(d, n, C.F32, C.ZVC)
+    for _ in range(3):
+        C.swap_out(d, n, C.F32, C.RLE).close()
+    live.wait()
+    C.release_cached(0)
+    assert live.host_bytes() == O.compress(x, O.ZVC, O.F32)
+    out = G.poisoned_words(n, 0)
+    live.swap_in(out)
+    live.wait()
+    assert np.array_equal(G.from_dev(out)[:n], x)
+    live.close()
+    h = C.swap_out(d, n, C.F32, C.ZVC)  # pools grow again after the release
+    h.wait()
+    assert h.host_bytes() == O.compress(x, O.ZVC, O.F32)
+    h.close()
