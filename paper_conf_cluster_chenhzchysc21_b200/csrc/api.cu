@@ -207,6 +207,13 @@ struct Ctx {
   cudaStream_t s_d2h = nullptr, s_h2d = nullptr, s_h2d2 = nullptr;
   cudaMemPool_t pool = nullptr;  // private stream-ordered pool (staging, LZ4 slots, decode scratch)
   uint64_t* dev_sink = nullptr;  // device word for container sizes nobody reads
+  // kernel-timing stamps (cswap_set_kernel_timing): a ring of 3-word slots in DEVICE memory.  A
+  // kernel that writes host-mapped memory while a copy streams over PCIe cannot complete until
+  // its write drains behind the copy's (~20-25 us, tools/event_gap_probe.cu), so stamps there
+  // would inflate the very duration they measure
+  static constexpr uint32_t kStampSlots = 1u << 14;
+  uint64_t* dev_stamps = nullptr;
+  std::atomic<uint32_t> stamp_next{0};
   // swap target (cswap_set_swap_target): -1 = pinned host; else a device whose memory holds the
   // containers (tpool: a pool located on that device, accessible from this one)
   int target = -1;
@@ -233,7 +240,7 @@ struct Ctx {
   struct Pend {
     cudaEvent_t a, b;
     cswap_kernel_record r;
-    uint64_t* stamps;  // 2 x u64 %globaltimer + the container size (mapped pinned), or null
+    uint64_t* stamps;  // device slot: 2 x u64 %globaltimer + the container size, or null
   };
   std::vector<Pend> pend;
 };
@@ -248,9 +255,11 @@ struct Timer {
   cudaStream_t st;
   cudaEvent_t a = nullptr, b = nullptr;
   bool started = false;
-  // [0], [1]: filled by stamp kernels first / last in the group (run_group); [2]: a swap-out's
-  // compress writes its container size here (read at collection time)
+  // device slot — [0], [1]: filled by stamp kernels first / last in the group (run_group; the first
+  // also clears [1] and [2]); [2]: a swap-out's compress writes its container size here (all
+  // three are read at collection time)
   uint64_t* stamps = nullptr;
+  bool stamped = false;  // a group's stamp kernels were enqueued (else the slot holds stale words)
   Timer(Ctx* ctx, cudaStream_t s);
   void start_now() {
     if (a && !started) {
@@ -267,7 +276,7 @@ struct Timer {
     if (!a) return;
     stop();
     std::lock_guard<std::mutex> lk(c->tm_m);
-    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0, 0.0}, stamps});
+    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0, 0.0}, stamped ? stamps : nullptr});
     a = b = nullptr;
     stamps = nullptr;
   }
@@ -279,15 +288,13 @@ namespace {
 Timer::Timer(Ctx* ctx, cudaStream_t s) : c(ctx), st(s) {
   if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) {
     t_pending = this;
-    stamps = reinterpret_cast<uint64_t*>(c->small.alloc(24));
-    if (stamps) stamps[0] = stamps[1] = stamps[2] = 0;
+    if (c->dev_stamps) stamps = c->dev_stamps + 3ull * (c->stamp_next.fetch_add(1) % Ctx::kStampSlots);
   }
 }
 Timer::~Timer() {
   if (t_pending == this) t_pending = nullptr;
   if (a) cudaEventDestroy(a);
   if (b) cudaEventDestroy(b);
-  if (stamps) c->small.free(reinterpret_cast<uint8_t*>(stamps));  // not committed
 }
 }  // namespace
 
@@ -353,12 +360,13 @@ cswap_status run_group(Ctx* c, cudaStream_t st, uint64_t key, Fn&& fn) {
   auto body = [&](cudaStream_t gs) -> cswap_status {
     if (stamps) {
       c->launches++;
-      TRY(cuda_status(launch_stamp(stamps, gs), "stamp"));
+      TRY(cuda_status(launch_stamp(stamps, gs, true), "stamp"));
+      pending->stamped = true;
     }
     TRY(fn(gs));
     if (stamps) {
       c->launches++;
-      TRY(cuda_status(launch_stamp(stamps + 1, gs), "stamp"));
+      TRY(cuda_status(launch_stamp(stamps + 1, gs, false), "stamp"));
     }
     return CSWAP_OK;
   };
@@ -1067,6 +1075,7 @@ cswap_status cswap_init(int device) {
   CU(cudaMalloc(&c->dev_err, 64));
   CU(cudaMemset(c->dev_err, 0, 64));
   CU(cudaMalloc(&c->dev_sink, 64));
+  CU(cudaMalloc(&c->dev_stamps, 3ull * 8 * Ctx::kStampSlots));
   if (const char* e = getenv("CSWAP_PINNED_CHUNK_MB")) c->pinned.chunk_bytes = uint64_t(atoll(e)) << 20;
   c->small.chunk_bytes = uint64_t(1) << 20;
   c->calib = builtin_calib();
@@ -1101,6 +1110,7 @@ cswap_status cswap_shutdown(void) {
   }
   cudaFree(c->dev_err);
   cudaFree(c->dev_sink);
+  cudaFree(c->dev_stamps);
   cudaMemPoolDestroy(c->pool);
   if (c->tpool) cudaMemPoolDestroy(c->tpool);
   cudaStreamDestroy(c->s_d2h);
@@ -1780,11 +1790,10 @@ uint64_t cswap_collect_kernel_timing(cswap_kernel_record* out, uint64_t cap) {
     cudaEventSynchronize(e.b);
     cudaEventElapsedTime(&ms, e.a, e.b);
     e.r.ms = ms;
-    if (e.stamps) {  // written by the group's stamp kernels, complete once e.b is
-      const volatile uint64_t* t = e.stamps;
+    uint64_t t[3] = {0, 0, 0};  // written by the group's stamp kernels, complete once e.b is
+    if (e.stamps && cudaMemcpy(t, e.stamps, sizeof(t), cudaMemcpyDeviceToHost) == cudaSuccess) {
       e.r.device_ms = (t[0] && t[1] > t[0]) ? double(t[1] - t[0]) * 1e-6 : 0.0;
       if (!e.r.comp_bytes) e.r.comp_bytes = t[2];  // swap-out compress: container size
-      c->small.free(reinterpret_cast<uint8_t*>(e.stamps));
     }
     if (out && k < cap) out[k] = e.r;
     k++;

@@ -212,15 +212,17 @@ cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtyp
   return cudaGetLastError();
 }
 
-// ---- timing stamps: one thread writes %globaltimer (ns) --------------------------------------
-__global__ void stamp_kernel(unsigned long long* dst) {
+// ---- timing stamps: one thread writes %globaltimer (ns) into a device slot; the group's first
+// stamp also clears the slot's end stamp and container-size word (slots are reused)
+__global__ void stamp_kernel(unsigned long long* dst, int first) {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  *dst = t;
+  dst[0] = t;
+  if (first) dst[1] = dst[2] = 0;
 }
 
-cudaError_t launch_stamp(uint64_t* dst, cudaStream_t st) {
-  stamp_kernel<<<1, 1, 0, st>>>(reinterpret_cast<unsigned long long*>(dst));
+cudaError_t launch_stamp(uint64_t* dst, cudaStream_t st, bool first) {
+  stamp_kernel<<<1, 1, 0, st>>>(reinterpret_cast<unsigned long long*>(dst), first ? 1 : 0);
   return cudaGetLastError();
 }
 

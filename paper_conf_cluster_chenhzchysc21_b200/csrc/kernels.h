@@ -23,7 +23,7 @@ cudaError_t launch_finalize(uint8_t* out, int codec, int dtype, uint64_t n, uint
                             const Scratch& sc, uint64_t* out_size, cudaStream_t st);
 cudaError_t launch_err_merge(const uint32_t* src, uint32_t* dst, cudaStream_t st);
 // one thread writes %globaltimer (ns) to dst (device-visible; here mapped pinned memory)
-cudaError_t launch_stamp(uint64_t* dst, cudaStream_t st);
+cudaError_t launch_stamp(uint64_t* dst, cudaStream_t st, bool first);
 cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, int dtype, uint8_t* out,
                                  uint64_t* out_size, cudaStream_t st);
 cudaError_t launch_none_decompress(const uint8_t* in, void* out, uint64_t n, int w, uint64_t F, const Scratch& sc,
