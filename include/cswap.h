@@ -230,12 +230,15 @@ cswap_status cswap_fit_linear(const double* X, const double* y, uint64_t m, uint
  * unknown), ms = CUDA-event time on the launch stream; device_ms = %globaltimer difference
  * between two 1-thread stamp kernels placed first and last in the group's graph (the group's
  * own device duration, without the event records' waits behind concurrent PCIe traffic;
- * 0 if unavailable). */
+ * 0 if unavailable); kernel_ms = the persistent ZVC compress kernel's own %globaltimer span,
+ * from the first CTA's start to the last CTA's finish before any host-memory store (0 for other
+ * groups). */
 typedef struct {
   int32_t codec, direction;
   uint64_t raw_bytes, comp_bytes;
   double ms;
   double device_ms;
+  double kernel_ms;
 } cswap_kernel_record;
 /* When enabled, the swap pipeline brackets its probe / compress / decompress launches with CUDA
  * events on the stream they are launched on. */

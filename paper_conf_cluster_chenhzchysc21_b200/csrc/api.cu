@@ -211,7 +211,7 @@ struct Ctx {
   // kernel that writes host-mapped memory while a copy streams over PCIe cannot complete until
   // its write drains behind the copy's (~20-25 us, tools/event_gap_probe.cu), so stamps there
   // would inflate the very duration they measure
-  static constexpr uint32_t kStampSlots = 1u << 14;
+  static constexpr uint32_t kStampSlots = 1u << 14, kStampWords = 5;
   uint64_t* dev_stamps = nullptr;
   std::atomic<uint32_t> stamp_next{0};
   // swap target (cswap_set_swap_target): -1 = pinned host; else a device whose memory holds the
@@ -240,7 +240,7 @@ struct Ctx {
   struct Pend {
     cudaEvent_t a, b;
     cswap_kernel_record r;
-    uint64_t* stamps;  // device slot: 2 x u64 %globaltimer + the container size, or null
+    uint64_t* stamps;  // device slot: 2 x u64 %globaltimer, the container size, kernel clock[2]; or null
   };
   std::vector<Pend> pend;
 };
@@ -276,7 +276,7 @@ struct Timer {
     if (!a) return;
     stop();
     std::lock_guard<std::mutex> lk(c->tm_m);
-    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0, 0.0}, stamped ? stamps : nullptr});
+    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0, 0.0, 0.0}, stamped ? stamps : nullptr});
     a = b = nullptr;
     stamps = nullptr;
   }
@@ -288,7 +288,8 @@ namespace {
 Timer::Timer(Ctx* ctx, cudaStream_t s) : c(ctx), st(s) {
   if (c->timing.load() && cudaEventCreate(&a) == cudaSuccess) {
     t_pending = this;
-    if (c->dev_stamps) stamps = c->dev_stamps + 3ull * (c->stamp_next.fetch_add(1) % Ctx::kStampSlots);
+    if (c->dev_stamps)
+      stamps = c->dev_stamps + uint64_t(Ctx::kStampWords) * (c->stamp_next.fetch_add(1) % Ctx::kStampSlots);
   }
 }
 Timer::~Timer() {
@@ -640,10 +641,12 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       // the end instead (no extra launch)
       static const bool end_kernel = getenv("CSWAP_ZVC_ENDPUB") && getenv("CSWAP_ZVC_ENDPUB")[0] == '0';  // A/B
       const uint32_t mode = frame_publish ? 1 : (end_kernel ? 0 : 2);
+      Scratch sc = mode ? with_prog(L.b->sc, mode) : L.b->sc;
+      // a timed group: the kernel also clocks itself into the timer's device slot (words 3, 4)
+      sc.kclock = (t_pending && t_pending->stamps) ? t_pending->stamps + 3 : nullptr;
       return run_group(c, st, group_key(kGrpCompress, codec, dtype) | (mode == 0 && prog ? 1u << 21 : 0u),
                        [&](cudaStream_t gs) {
-                         TRY(cuda_status(launch_zvc_compress(in, n, w, F, out, out_size,
-                                                             mode ? with_prog(L.b->sc, mode) : L.b->sc, ep, dtype, gs),
+                         TRY(cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, sc, ep, dtype, gs),
                                          "zvc_compress"));
                          return mode == 0 ? publish(gs) : CSWAP_OK;
                        });
@@ -1075,7 +1078,7 @@ cswap_status cswap_init(int device) {
   CU(cudaMalloc(&c->dev_err, 64));
   CU(cudaMemset(c->dev_err, 0, 64));
   CU(cudaMalloc(&c->dev_sink, 64));
-  CU(cudaMalloc(&c->dev_stamps, 3ull * 8 * Ctx::kStampSlots));
+  CU(cudaMalloc(&c->dev_stamps, 8ull * Ctx::kStampWords * Ctx::kStampSlots));
   if (const char* e = getenv("CSWAP_PINNED_CHUNK_MB")) c->pinned.chunk_bytes = uint64_t(atoll(e)) << 20;
   c->small.chunk_bytes = uint64_t(1) << 20;
   c->calib = builtin_calib();
@@ -1790,10 +1793,11 @@ uint64_t cswap_collect_kernel_timing(cswap_kernel_record* out, uint64_t cap) {
     cudaEventSynchronize(e.b);
     cudaEventElapsedTime(&ms, e.a, e.b);
     e.r.ms = ms;
-    uint64_t t[3] = {0, 0, 0};  // written by the group's stamp kernels, complete once e.b is
+    uint64_t t[Ctx::kStampWords] = {};  // written by the group's kernels, complete once e.b is
     if (e.stamps && cudaMemcpy(t, e.stamps, sizeof(t), cudaMemcpyDeviceToHost) == cudaSuccess) {
       e.r.device_ms = (t[0] && t[1] > t[0]) ? double(t[1] - t[0]) * 1e-6 : 0.0;
       if (!e.r.comp_bytes) e.r.comp_bytes = t[2];  // swap-out compress: container size
+      e.r.kernel_ms = (t[3] != ~0ull && t[4] > t[3]) ? double(t[4] - t[3]) * 1e-6 : 0.0;
     }
     if (out && k < cap) out[k] = e.r;
     k++;

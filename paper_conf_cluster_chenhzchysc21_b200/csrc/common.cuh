@@ -47,7 +47,16 @@ struct Scratch {
   // ZVC compress only: 1 = publish each frame as soon as it is complete (the producer warps),
   // 2 = the last CTA publishes every frame once the kernel is done (no extra launch)
   uint32_t prog_mode;
+  // kernel timing (NULL unless cswap_set_kernel_timing): device u64[2] = {min CTA start,
+  // end} in %globaltimer ns, written by the persistent ZVC compress (slot [0] preset to ~0)
+  uint64_t* kclock;
 };
+
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 constexpr uint64_t kProgReady = 1ull << 63;
 
 // Publish "frame k complete, ends at byte `end`" to host-mapped memory.  The caller has made the

@@ -218,7 +218,10 @@ __global__ void stamp_kernel(unsigned long long* dst, int first) {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   dst[0] = t;
-  if (first) dst[1] = dst[2] = 0;
+  if (first) {  // slot: [0] start, [1] end, [2] container size, [3..4] kernel clock (Scratch::kclock)
+    dst[1] = dst[2] = dst[4] = 0;
+    dst[3] = ~0ull;
+  }
 }
 
 cudaError_t launch_stamp(uint64_t* dst, cudaStream_t st, bool first) {

@@ -205,6 +205,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) {
+    if (sc.kclock) atomicMin(reinterpret_cast<unsigned long long*>(sc.kclock), (unsigned long long)globaltimer_ns());
     for (int s = 0; s < S; s++) {
       mbar_init(&bar_full[s], 1);
       mbar_init(&bar_empty[s], CW);
@@ -598,6 +599,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
   }
   __syncthreads();
   if (s_last) {
+    if (sc.kclock && tid == 0) sc.kclock[1] = globaltimer_ns();  // before the host-memory stores below
     for (uint64_t q = tid; q < nacc; q += blockDim.x) sc.zacc[q] = 0;
     if (tid == 0) sc.zacc[nacc] = 0;
     // swap-out progress published at the end (prog_mode 2): every tile of every CTA is emitted

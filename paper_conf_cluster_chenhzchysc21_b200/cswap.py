@@ -74,7 +74,8 @@ class Decision(ctypes.Structure):
 
 class KernelRecord(ctypes.Structure):
     _fields_ = [("codec", ctypes.c_int32), ("direction", ctypes.c_int32), ("raw_bytes", ctypes.c_uint64),
-                ("comp_bytes", ctypes.c_uint64), ("ms", ctypes.c_double), ("device_ms", ctypes.c_double)]
+                ("comp_bytes", ctypes.c_uint64), ("ms", ctypes.c_double), ("device_ms", ctypes.c_double),
+                ("kernel_ms", ctypes.c_double)]
 
 
 _vp, _u64, _u32, _i, _d = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int, ctypes.c_double
@@ -349,7 +350,7 @@ def collect_kernel_timing(cap: int = 1 << 16):
     buf = (KernelRecord * cap)()
     k = int(_L.cswap_collect_kernel_timing(buf, cap))
     return [{"codec": r.codec, "direction": r.direction, "raw_bytes": r.raw_bytes, "comp_bytes": r.comp_bytes,
-             "ms": r.ms, "device_ms": r.device_ms} for r in buf[:k]]
+             "ms": r.ms, "device_ms": r.device_ms, "kernel_ms": r.kernel_ms} for r in buf[:k]]
 
 
 def kernel_launches() -> int:
