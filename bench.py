@@ -366,8 +366,8 @@ def _roofline(records, steps: int = 1) -> dict:
         out["kernel_clock"] = {
             "achieved": round(kc, 1), "frac": round(kc / peak, 4), "avg_launch_ms": round(g["k_ms"] / g["launches"], 4),
             "how": "same launches, same bytes; duration = the persistent compress kernel's own %globaltimer span "
-                   "(first CTA's start, atomicMin, to the last CTA's finish, before its host-memory stores), "
-                   "written to device memory"}
+                   "(CTA 0's start to the last CTA's finish, before its host-memory stores; the grid is co-resident), "
+                   "written to device memory; the timed compress groups carry no stamp kernels"}
     out["all_kernels"] = {f"{names[c]}_{'c' if dd == 0 else 'dc'}": {
         "GBps": round(v["bytes"] / (v["ms"] * 1e-3) / 1e9, 1), "frac": round(v["bytes"] / (v["ms"] * 1e-3) / 1e9 / peak, 4),
         "ms_total": round(v["ms"], 3), "launches": v["launches"]} for (c, dd), v in groups.items()}

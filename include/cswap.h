@@ -231,8 +231,8 @@ cswap_status cswap_fit_linear(const double* X, const double* y, uint64_t m, uint
  * between two 1-thread stamp kernels placed first and last in the group's graph (the group's
  * own device duration, without the event records' waits behind concurrent PCIe traffic;
  * 0 if unavailable); kernel_ms = the persistent ZVC compress kernel's own %globaltimer span,
- * from the first CTA's start to the last CTA's finish before any host-memory store (0 for other
- * groups). */
+ * from CTA 0's start to the last CTA's finish before any host-memory store (0 for other groups;
+ * such a group has no stamp kernels, so its device_ms is 0). */
 typedef struct {
   int32_t codec, direction;
   uint64_t raw_bytes, comp_bytes;

@@ -241,6 +241,7 @@ struct Ctx {
     cudaEvent_t a, b;
     cswap_kernel_record r;
     uint64_t* stamps;  // device slot: 2 x u64 %globaltimer, the container size, kernel clock[2]; or null
+    bool stamped, self_clocked;  // which words of the slot this group wrote
   };
   std::vector<Pend> pend;
 };
@@ -259,7 +260,10 @@ struct Timer {
   // also clears [1] and [2]); [2]: a swap-out's compress writes its container size here (all
   // three are read at collection time)
   uint64_t* stamps = nullptr;
-  bool stamped = false;  // a group's stamp kernels were enqueued (else the slot holds stale words)
+  bool stamped = false;  // a group's stamp kernels were enqueued (else words 0, 1 are stale)
+  // the group's kernel clocks itself (words 3, 4) and writes the container size (word 2): no stamp
+  // kernels, whose boundaries cost ~12 us each while a copy streams
+  bool self_clocked = false;
   Timer(Ctx* ctx, cudaStream_t s);
   void start_now() {
     if (a && !started) {
@@ -276,7 +280,8 @@ struct Timer {
     if (!a) return;
     stop();
     std::lock_guard<std::mutex> lk(c->tm_m);
-    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0, 0.0, 0.0}, stamped ? stamps : nullptr});
+    c->pend.push_back(Ctx::Pend{a, b, cswap_kernel_record{codec, dir, raw, comp, 0.0, 0.0, 0.0},
+                                (stamped || self_clocked) ? stamps : nullptr, stamped, self_clocked});
     a = b = nullptr;
     stamps = nullptr;
   }
@@ -356,7 +361,7 @@ constexpr size_t kGraphCacheMax = 64;
 template <class Fn>
 cswap_status run_group(Ctx* c, cudaStream_t st, uint64_t key, Fn&& fn) {
   Timer* pending = t_pending;
-  uint64_t* stamps = pending ? pending->stamps : nullptr;
+  uint64_t* stamps = pending && !pending->self_clocked ? pending->stamps : nullptr;
   // timed groups: stamp kernels first and last (device duration of the group)
   auto body = [&](cudaStream_t gs) -> cswap_status {
     if (stamps) {
@@ -643,7 +648,11 @@ cswap_status do_compress(Ctx* c, const void* in, uint64_t n, int dtype, int code
       const uint32_t mode = frame_publish ? 1 : (end_kernel ? 0 : 2);
       Scratch sc = mode ? with_prog(L.b->sc, mode) : L.b->sc;
       // a timed group: the kernel also clocks itself into the timer's device slot (words 3, 4)
-      sc.kclock = (t_pending && t_pending->stamps) ? t_pending->stamps + 3 : nullptr;
+      sc.kclock = nullptr;
+      if (t_pending && t_pending->stamps) {
+        sc.kclock = t_pending->stamps + 3;
+        t_pending->self_clocked = true;
+      }
       return run_group(c, st, group_key(kGrpCompress, codec, dtype) | (mode == 0 && prog ? 1u << 21 : 0u),
                        [&](cudaStream_t gs) {
                          TRY(cuda_status(launch_zvc_compress(in, n, w, F, out, out_size, sc, ep, dtype, gs),
@@ -1795,9 +1804,9 @@ uint64_t cswap_collect_kernel_timing(cswap_kernel_record* out, uint64_t cap) {
     e.r.ms = ms;
     uint64_t t[Ctx::kStampWords] = {};  // written by the group's kernels, complete once e.b is
     if (e.stamps && cudaMemcpy(t, e.stamps, sizeof(t), cudaMemcpyDeviceToHost) == cudaSuccess) {
-      e.r.device_ms = (t[0] && t[1] > t[0]) ? double(t[1] - t[0]) * 1e-6 : 0.0;
+      if (e.stamped) e.r.device_ms = (t[0] && t[1] > t[0]) ? double(t[1] - t[0]) * 1e-6 : 0.0;
+      if (e.self_clocked) e.r.kernel_ms = t[4] > t[3] ? double(t[4] - t[3]) * 1e-6 : 0.0;
       if (!e.r.comp_bytes) e.r.comp_bytes = t[2];  // swap-out compress: container size
-      e.r.kernel_ms = (t[3] != ~0ull && t[4] > t[3]) ? double(t[4] - t[3]) * 1e-6 : 0.0;
     }
     if (out && k < cap) out[k] = e.r;
     k++;

@@ -47,8 +47,8 @@ struct Scratch {
   // ZVC compress only: 1 = publish each frame as soon as it is complete (the producer warps),
   // 2 = the last CTA publishes every frame once the kernel is done (no extra launch)
   uint32_t prog_mode;
-  // kernel timing (NULL unless cswap_set_kernel_timing): device u64[2] = {min CTA start,
-  // end} in %globaltimer ns, written by the persistent ZVC compress (slot [0] preset to ~0)
+  // kernel timing (NULL unless cswap_set_kernel_timing): device u64[2] = {CTA 0's start, the
+  // last CTA's finish} in %globaltimer ns, written by the persistent ZVC compress
   uint64_t* kclock;
 };
 

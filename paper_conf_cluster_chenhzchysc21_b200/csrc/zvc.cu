@@ -205,7 +205,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) {
-    if (sc.kclock) atomicMin(reinterpret_cast<unsigned long long*>(sc.kclock), (unsigned long long)globaltimer_ns());
+    if (sc.kclock && blockIdx.x == 0) sc.kclock[0] = globaltimer_ns();  // the grid is co-resident (cooperative)
     for (int s = 0; s < S; s++) {
       mbar_init(&bar_full[s], 1);
       mbar_init(&bar_empty[s], CW);
