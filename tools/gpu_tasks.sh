@@ -15,7 +15,8 @@
 #   calibrate  re-fit calib/b200.json on the box (bench.py --calibrate)
 #   next       NEXT-row measurements: launch_tune, time models, drift, training steps
 #   pipeline   swap pipeline timeline / granularity probe (tools/pipeline_probe.py)
-#   probes     event cost during copies, D2H rates by allocation, SM-driven vs copy-engine copies
+#   probes     event cost during copies (event_probe, event_gap_probe), D2H rates by allocation,
+#              SM-driven vs copy-engine copies, host time of small codec calls, link ramp on a box
 #   cpuplan    oracle CPU timing plan (bench.py --cpu-plan)
 mkdir -p gpurun_out
 R=/tmp/ncu_reps; mkdir -p $R
@@ -82,7 +83,10 @@ for task in "$@"; do
   probes)
     nvcc -gencode arch=compute_100a,code=sm_100a -O2 -o /tmp/evp tools/event_probe.cu && timeout 300 /tmp/evp > gpurun_out/event_probe.jsonl 2>&1
     nvcc -gencode arch=compute_100a,code=sm_100a -O2 -o /tmp/d2hp tools/d2h_probe.cu && timeout 300 /tmp/d2hp > gpurun_out/d2h_probe.jsonl 2>&1
-    nvcc -gencode arch=compute_100a,code=sm_100a -O3 -shared -Xcompiler -fPIC tools/zc_probe.cu -o tools/zc_probe.so && timeout 300 python tools/zc_probe.py > gpurun_out/zc_probe.txt 2>&1 ;;
+    nvcc -gencode arch=compute_100a,code=sm_100a -O3 -shared -Xcompiler -fPIC tools/zc_probe.cu -o tools/zc_probe.so && timeout 300 python tools/zc_probe.py > gpurun_out/zc_probe.txt 2>&1
+    nvcc -gencode arch=compute_100a,code=sm_100a -O2 -o /tmp/egp tools/event_gap_probe.cu && timeout 300 /tmp/egp > gpurun_out/event_gap_probe.txt 2>&1
+    timeout 300 python tools/host_overhead_probe.py > gpurun_out/host_overhead.jsonl 2>&1
+    timeout 120 python tools/fresh_box_probe.py > gpurun_out/fresh_box_probe.jsonl 2>&1 ;;
   cpuplan)
     timeout 1800 python bench.py --cpu-plan gpurun_out/cpu_plan.json > gpurun_out/cpu_plan.log 2>&1 ;;
   *) echo "unknown task $task" ;;
