@@ -17,9 +17,12 @@ from paper_conf_cluster_chenhzchysc21_b200 import calibrate, cswap as C  # noqa:
 C.init(0)
 calibrate.load(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), 'calib', 'b200.json'))
 ts, outs, ns = [], [], []
-for i, (name, shape, s) in enumerate(synth.vgg16_b64()):
+# PROBE_WORKLOAD = vgg16 (default) | resnet50 | bert: bench.py's sets and dtypes
+WL = os.environ.get('PROBE_WORKLOAD', 'vgg16')
+SPEC, DT = {'vgg16': (synth.vgg16_b64, 0), 'resnet50': (synth.resnet50_b64, 0), 'bert': (synth.bert_large_b8, 1)}[WL]
+for i, (name, shape, s) in enumerate(SPEC()):
     n = synth.numel(shape)
-    ts.append(synth.relu_iid_torch(n, s, seed=synth.seed_of(3, 0, 0, i), dtype=0, device='cuda'))
+    ts.append(synth.relu_iid_torch(n, s, seed=synth.seed_of(3, 0, 0, i), dtype=DT, device='cuda'))
     outs.append(torch.empty_like(ts[-1]))
     ns.append(n)
 codec = int(sys.argv[1]) if len(sys.argv) > 1 else C.AUTO
@@ -43,9 +46,9 @@ def step():
         hs = []
         for t, n, e in zip(ts, ns, landed):
             st.wait_event(e)
-            hs.append(C.swap_out(t, n, 0, codec))
+            hs.append(C.swap_out(t, n, DT, codec))
     else:
-        hs = [C.swap_out(t, n, 0, codec) for t, n in zip(ts, ns)]
+        hs = [C.swap_out(t, n, DT, codec) for t, n in zip(ts, ns)]
     for o, h in zip(reversed(outs), reversed(hs)):
         h.swap_in(o)
     return hs
