@@ -154,6 +154,44 @@ __device__ __forceinline__ uint32_t mad_u32(uint32_t a, uint32_t c) {
   return r;
 }
 
+#ifndef CSWAP_ZVC_ROWASM
+#define CSWAP_ZVC_ROWASM 1
+#endif
+// One row of the compacting count: p = (x != 0); w = ballot(p); @p store x at the shared byte
+// address sdp + W * popc(w & lt); sdp += W * popc(w).  A single predicate register serves the
+// ballot and the store.
+template <typename T>
+__device__ __forceinline__ void row_compact(uint32_t x, uint32_t lt, uint32_t& sdp, uint32_t& w) {
+  if constexpr (sizeof(T) == 4) {
+    asm("{\n\t.reg .pred p;\n\t.reg .b32 r, a;\n\t"
+        "setp.ne.u32 p, %2, 0;\n\t"
+        "vote.sync.ballot.b32 %0, p, 0xffffffff;\n\t"
+        "and.b32 r, %0, %3;\n\t"
+        "popc.b32 r, r;\n\t"
+        "mad.lo.u32 a, r, 4, %1;\n\t"
+        "@p st.shared.u32 [a], %2;\n\t"
+        "popc.b32 r, %0;\n\t"
+        "mad.lo.u32 %1, r, 4, %1;\n\t}"
+        : "=&r"(w), "+r"(sdp)
+        : "r"(x), "r"(lt)
+        : "memory");
+  } else {
+    asm("{\n\t.reg .pred p;\n\t.reg .b32 r, a;\n\t.reg .b16 h;\n\t"
+        "setp.ne.u32 p, %2, 0;\n\t"
+        "vote.sync.ballot.b32 %0, p, 0xffffffff;\n\t"
+        "and.b32 r, %0, %3;\n\t"
+        "popc.b32 r, r;\n\t"
+        "mad.lo.u32 a, r, 2, %1;\n\t"
+        "cvt.u16.u32 h, %2;\n\t"
+        "@p st.shared.u16 [a], h;\n\t"
+        "popc.b32 r, %0;\n\t"
+        "mad.lo.u32 %1, r, 2, %1;\n\t}"
+        : "=&r"(w), "+r"(sdp)
+        : "r"(x), "r"(lt)
+        : "memory");
+  }
+}
+
 // compress tile geometry: TB bytes per tile
 template <typename T, int TB>
 struct CGeom {
@@ -445,7 +483,14 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       }
 #pragma unroll
       for (int u = 0; u < B; u++) {
-        const uint32_t w = __ballot_sync(0xffffffffu, v[u] != 0);
+        uint32_t w;
+        if (CSWAP_ZVC_ROWASM) {
+          // one predicate for the ballot and the store (written in C++, ptxas recomputes the
+          // row's predicate for the predicated store)
+          row_compact<T>(v[u], lt, sdp, w);
+        } else {
+          w = __ballot_sync(0xffffffffu, v[u] != 0);
+        }
         // bitmap words leave lane 0 four at a time (one 16-byte shared store per 4 rows)
         if (CSWAP_ZVC_BM4) {
           wq[u & 3] = w;
@@ -454,8 +499,10 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         } else if (lane == 0) {
           bm_out[m0 + u] = w;
         }
-        if (v[u]) sts_word<T>(mad_u32<G::W>(__popc(w & lt), sdp), v[u]);
-        sdp = mad_u32<G::W>(__popc(w), sdp);
+        if (!CSWAP_ZVC_ROWASM) {
+          if (v[u]) sts_word<T>(mad_u32<G::W>(__popc(w & lt), sdp), v[u]);
+          sdp = mad_u32<G::W>(__popc(w), sdp);
+        }
       }
       if (m0 + B < EROWS) {
         if (!CSWAP_ZVC_PF) {
