@@ -7,7 +7,7 @@ reverse order, H2D + decompress (swap-in) (Fig. 2, :64-:72; vDNN policy
 value = raw tensor bytes swapped out and back in per second, summed over ranks (GB/s).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--workload vgg16|resnet50|bert] [--calibrate] [--no-extras]
+                    [--workload vgg16|resnet50|resnet50_f16|bert] [--calibrate] [--no-extras]
 Multi-GPU ("replicas only"): one process per GPU, each swapping its own replica
 of the set (no collective on the data path, "scaling": "weak"); time = the slowest rank's device
 time.  Under torchrun the ranks come from the environment; `python bench.py --gpus N` without
@@ -43,6 +43,8 @@ def workload(name: str):
         return "vgg16_b64_swapset", synth.vgg16_b64(), synth.F32
     if name == "resnet50":
         return "resnet50_b64_swapset", synth.resnet50_b64(), synth.F32
+    if name == "resnet50_f16":  # BASELINE configs[3]: the same set in fp16 (1197.4 MiB)
+        return "resnet50_b64_f16_swapset", synth.resnet50_b64(), synth.F16
     if name == "bert":
         return "bert_large_b8_swapset", synth.bert_large_b8(), synth.F16
     raise SystemExit(f"unknown workload {name}")
@@ -869,7 +871,7 @@ def main(argv=None):
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="vgg16", choices=["vgg16", "resnet50", "bert"])
+    ap.add_argument("--workload", default="vgg16", choices=["vgg16", "resnet50", "resnet50_f16", "bert"])
     ap.add_argument("--calibrate", action="store_true", help="full calibration sweep, writes calib/b200.json")
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")

@@ -31,6 +31,7 @@ for task in "$@"; do
     timeout 900 python bench.py --steps 20 --warmup 5 > gpurun_out/b_bench.json 2> gpurun_out/b_bench.err
     timeout 900 python bench.py --workload bert --no-cpu > gpurun_out/b_bench_bert.json 2> gpurun_out/b_bench_bert.err
     timeout 900 python bench.py --workload resnet50 --no-cpu > gpurun_out/b_bench_resnet50.json 2> gpurun_out/b_bench_resnet50.err
+    timeout 900 python bench.py --workload resnet50_f16 --no-cpu > gpurun_out/b_bench_resnet50_f16.json 2> gpurun_out/b_bench_resnet50_f16.err
     timeout 900 python bench.py --impl reference --steps 20 --warmup 5 > gpurun_out/b_reference.json 2> gpurun_out/b_reference.err ;;
   zvc)
     out=gpurun_out/z_zvc.jsonl; : > $out

@@ -19,7 +19,8 @@ calibrate.load(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__fi
 ts, outs, ns = [], [], []
 # PROBE_WORKLOAD = vgg16 (default) | resnet50 | bert: bench.py's sets and dtypes
 WL = os.environ.get('PROBE_WORKLOAD', 'vgg16')
-SPEC, DT = {'vgg16': (synth.vgg16_b64, 0), 'resnet50': (synth.resnet50_b64, 0), 'bert': (synth.bert_large_b8, 1)}[WL]
+SPEC, DT = {'vgg16': (synth.vgg16_b64, 0), 'resnet50': (synth.resnet50_b64, 0), 'resnet50_f16': (synth.resnet50_b64, 1),
+            'bert': (synth.bert_large_b8, 1)}[WL]
 for i, (name, shape, s) in enumerate(SPEC()):
     n = synth.numel(shape)
     ts.append(synth.relu_iid_torch(n, s, seed=synth.seed_of(3, 0, 0, i), dtype=DT, device='cuda'))
