@@ -72,11 +72,24 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 template <int S, int CW>
 constexpr int compress_threads() { return 32 * (CW + 1 + S); }
 
-// resolver polling: __nanosleep backoff bounds (ns)
+// resolver polling: __nanosleep backoff bounds (ns).  A/B x2 of 32 / 16 / 8 ns / no sleep
+// (profiles/zvc_backoff_ab_r02.jsonl): 8 ns is fastest or tied everywhere (1 GiB f32 s = 0.5
+// 0.332 -> 0.326 ms, s = 0.8 0.303 -> 0.297; 256 MiB -2 %; f16 -0.5..1 %): a resolver that
+// learns a count sooner releases the consumers' emit sooner; spinning without a sleep takes
+// issue slots from the consumers (worse than 8 ns)
 #ifndef CSWAP_ZVC_MAX_BACKOFF
-#define CSWAP_ZVC_MAX_BACKOFF 32
+#define CSWAP_ZVC_MAX_BACKOFF 8
 #endif
-constexpr uint32_t kMinBackoff = 16, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
+#ifndef CSWAP_ZVC_MIN_BACKOFF
+#define CSWAP_ZVC_MIN_BACKOFF 8
+#endif
+constexpr uint32_t kMinBackoff = CSWAP_ZVC_MIN_BACKOFF, kMaxBackoff = CSWAP_ZVC_MAX_BACKOFF;
+// one resolver poll pause: __nanosleep with exponential backoff (kMaxBackoff = 0: spin)
+__device__ __forceinline__ void resolver_pause(uint32_t& backoff) {
+  if (kMaxBackoff == 0) return;
+  __nanosleep(backoff);
+  backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
+}
 // rows per batch of count_slab's loads
 #ifndef CSWAP_ZVC_POW2
 #define CSWAP_ZVC_POW2 1
@@ -359,15 +372,13 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           uint64_t a, acc;
           uint32_t backoff = kMinBackoff;
           while (status_flag(a = ld_relaxed(sc.aux + k - 1), epoch) != kFlagP) {
-            __nanosleep(backoff);
-            backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
+            resolver_pause(backoff);
           }
           const uint64_t Fp = frame_len(n, F, k - 1);
           const uint64_t tiles_prev = cdiv(Fp, G::TILE);
-          backoff = 32;
+          backoff = kMinBackoff;
           while (((acc = ld_relaxed(sc.zacc + k - 1)) >> 40) != tiles_prev) {
-            __nanosleep(backoff);
-            backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
+            resolver_pause(backoff);
           }
           fstart = status_value(a) + a16(4 * cdiv(Fp, 32)) + a16(G::W * (acc & ((1ull << 40) - 1)));
         }
@@ -383,8 +394,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
             const uint64_t* p = sc.zacc + K + uint64_t(k) * gpf + gi;
             uint32_t backoff = kMinBackoff;
             while (((v = ld_relaxed(p)) >> 40) != 32) {
-              __nanosleep(backoff);
-              backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
+              resolver_pause(backoff);
             }
             v &= (1ull << 40) - 1;
           }
@@ -397,8 +407,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           uint64_t st;
           uint32_t backoff = kMinBackoff;
           while (status_flag(st = ld_relaxed(p), epoch) == 0) {
-            __nanosleep(backoff);
-            backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
+            resolver_pause(backoff);
           }
           v = status_value(st);
         }
@@ -409,8 +418,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           uint64_t a;
           uint32_t backoff = kMinBackoff;
           while (status_flag(a = ld_relaxed(sc.aux + k), epoch) != kFlagP) {
-            __nanosleep(backoff);
-            backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
+            resolver_pause(backoff);
           }
           fstart = status_value(a);
         }
