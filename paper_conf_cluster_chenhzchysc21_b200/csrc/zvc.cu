@@ -91,6 +91,15 @@ __device__ __forceinline__ void resolver_pause(uint32_t& backoff) {
   backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
 }
 // rows per batch of count_slab's loads
+// accumulator words (per frame, per 32-tile group, per frame done-count, the CTA counter) are
+// CSWAP_ZVC_ACC_STRIDE u64 apart: 16 puts each on its own 128-byte line.  Packed, a frame's 16
+// group words shared one line that every consumer's atomics and every resolver's polls hit;
+// A/B x2 (profiles/zvc_accstride_ab_r02.jsonl): 1 GiB f32 0.328 -> 0.322 ms (s = 0.5), 0.301 ->
+// 0.293 (s = 0.8), 0.291 -> 0.283 (s = 0.95); 96 / 256 MiB f32 -2..4 %; 16-bit unchanged
+#ifndef CSWAP_ZVC_ACC_STRIDE
+#define CSWAP_ZVC_ACC_STRIDE 16
+#endif
+constexpr uint64_t kAccStride = CSWAP_ZVC_ACC_STRIDE;
 #ifndef CSWAP_ZVC_POW2
 #define CSWAP_ZVC_POW2 1
 #endif
@@ -283,7 +292,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
     // acquire.cta), count it for its frame with a gpu-scope acq_rel atomic; the CTA that
     // completes a frame publishes the frame's end offset (frame start + its frame-table entry,
     // both written before the frame's last tiles were emitted) for the host's per-frame D2H
-    uint64_t* const fdone = sc.zacc + K + uint64_t(K) * gpf;  // after the accumulators
+    uint64_t* const fdone = sc.zacc + (K + uint64_t(K) * gpf) * kAccStride;  // after the accumulators
     auto tile_emitted = [&](uint32_t t) {
       if (!sc.prog || sc.prog_mode != 1 || lane != 0) return;
       uint32_t k, j, te, be;
@@ -292,7 +301,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       unsigned long long old;
       asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;"
                    : "=l"(old)
-                   : "l"(fdone + k)
+                   : "l"(fdone + k * kAccStride)
                    : "memory");
       if (old + 1 == cdiv(Fk, G::TILE)) {
         const uint64_t fs = status_value(ld_relaxed(sc.aux + k));
@@ -377,7 +386,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           const uint64_t Fp = frame_len(n, F, k - 1);
           const uint64_t tiles_prev = cdiv(Fp, G::TILE);
           backoff = kMinBackoff;
-          while (((acc = ld_relaxed(sc.zacc + k - 1)) >> 40) != tiles_prev) {
+          while (((acc = ld_relaxed(sc.zacc + (k - 1) * kAccStride)) >> 40) != tiles_prev) {
             resolver_pause(backoff);
           }
           fstart = status_value(a) + a16(4 * cdiv(Fp, 32)) + a16(G::W * (acc & ((1ull << 40) - 1)));
@@ -391,7 +400,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
           const uint32_t gi = g0 + lane;
           uint64_t v = 0;
           if (gi < g) {
-            const uint64_t* p = sc.zacc + K + uint64_t(k) * gpf + gi;
+            const uint64_t* p = sc.zacc + (K + uint64_t(k) * gpf + gi) * kAccStride;
             uint32_t backoff = kMinBackoff;
             while (((v = ld_relaxed(p)) >> 40) != 32) {
               resolver_pause(backoff);
@@ -548,8 +557,9 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
 #pragma unroll
       for (int w = 0; w < CW; w++) tot += s_wtot[s][w];
       st_relaxed(sc.status + t, make_status(tot, epoch, kFlagA));  // self-contained: no release needed
-      atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + k), (1ull << 40) + tot);
-      atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + K + uint64_t(k) * gpf + j / 32), (1ull << 40) + tot);
+      atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + k * kAccStride), (1ull << 40) + tot);
+      atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + (K + uint64_t(k) * gpf + j / 32) * kAccStride),
+                (1ull << 40) + tot);
       s_nnz[s] = tot;
       if (!kNamedBars) mbar_arrive(&bar_cnt[s]);
     }
@@ -649,14 +659,14 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
   const uint64_t nacc = 2 * uint64_t(K) + uint64_t(K) * gpf;
   if (tid == 0) {
     unsigned long long old;
-    asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;" : "=l"(old) : "l"(sc.zacc + nacc) : "memory");
+    asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;" : "=l"(old) : "l"(sc.zacc + nacc * kAccStride) : "memory");
     s_last = old + 1 == gridDim.x;
   }
   __syncthreads();
   if (s_last) {
     if (sc.kclock && tid == 0) sc.kclock[1] = globaltimer_ns();  // before the host-memory stores below
-    for (uint64_t q = tid; q < nacc; q += blockDim.x) sc.zacc[q] = 0;
-    if (tid == 0) sc.zacc[nacc] = 0;
+    for (uint64_t q = tid; q < nacc; q += blockDim.x) sc.zacc[q * kAccStride] = 0;
+    if (tid == 0) sc.zacc[nacc * kAccStride] = 0;
     // swap-out progress published at the end (prog_mode 2): every tile of every CTA is emitted
     // (each CTA's done-count release covers its stores; this CTA acquired all of them), so the
     // frame starts and frame-table entries are final
@@ -1071,7 +1081,8 @@ static cudaError_t launch_compress_t(const void* in, uint64_t n, uint64_t F, uin
 void zvc_compress_scratch(uint64_t n, int w, uint64_t F, uint64_t* tiles, uint64_t* aux) {
   const uint64_t TILE = 16384 / w, K = cdiv(n, F), tpf = cdiv(F, TILE);
   *tiles = K ? (K - 1) * tpf + cdiv(frame_len(n, F, K - 1), TILE) : 0;
-  *aux = 2 * K + K * ((tpf + 31) / 32) + 2;  // sc.zacc: frame + group accumulators, fdone, CTA counter
+  // sc.zacc: frame + group accumulators, fdone, CTA counter, kAccStride words apart
+  *aux = (2 * K + K * ((tpf + 31) / 32) + 2) * kAccStride;
 }
 
 cudaError_t launch_zvc_compress(const void* in, uint64_t n, int w, uint64_t F, uint8_t* out, uint64_t* out_size,
