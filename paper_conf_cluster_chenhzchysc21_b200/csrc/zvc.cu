@@ -100,6 +100,15 @@ __device__ __forceinline__ void resolver_pause(uint32_t& backoff) {
 #define CSWAP_ZVC_ACC_STRIDE 16
 #endif
 constexpr uint64_t kAccStride = CSWAP_ZVC_ACC_STRIDE;
+// tile status words CSWAP_ZVC_STATUS_STRIDE u64 apart: each tile's count is stored once by its
+// CTA and polled by the resolvers of the later tiles of its group; packed four to a 32-byte
+// sector, neighbouring CTAs' stores and those polls met on the same sectors.  A/B x2
+// (profiles/zvc_statusstride_ab_r02.jsonl): stride 2 and 16 equal, 1 GiB f32 0.320 -> 0.309 ms
+// (s = 0.5), 0.281 -> 0.276 (s = 0.95), 96 / 256 MiB f32 -2..5 %, f16 -0.5..1 %
+#ifndef CSWAP_ZVC_STATUS_STRIDE
+#define CSWAP_ZVC_STATUS_STRIDE 2
+#endif
+constexpr uint64_t kStatusStride = CSWAP_ZVC_STATUS_STRIDE;
 #ifndef CSWAP_ZVC_POW2
 #define CSWAP_ZVC_POW2 1
 #endif
@@ -412,7 +421,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
         const uint32_t jj = j - 32 * g;  // earlier tiles of this group
         uint64_t v = 0;
         if (uint32_t(lane) < jj) {
-          const uint64_t* p = sc.status + (t - jj + lane);
+          const uint64_t* p = sc.status + uint64_t(t - jj + lane) * kStatusStride;
           uint64_t st;
           uint32_t backoff = kMinBackoff;
           while (status_flag(st = ld_relaxed(p), epoch) == 0) {
@@ -556,7 +565,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       uint32_t tot = 0;
 #pragma unroll
       for (int w = 0; w < CW; w++) tot += s_wtot[s][w];
-      st_relaxed(sc.status + t, make_status(tot, epoch, kFlagA));  // self-contained: no release needed
+      st_relaxed(sc.status + uint64_t(t) * kStatusStride, make_status(tot, epoch, kFlagA));  // self-contained: no release needed
       atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + k * kAccStride), (1ull << 40) + tot);
       atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + (K + uint64_t(k) * gpf + j / 32) * kAccStride),
                 (1ull << 40) + tot);
@@ -1080,7 +1089,7 @@ static cudaError_t launch_compress_t(const void* in, uint64_t n, uint64_t F, uin
 // sized for the smallest compress tile any configuration uses (16 KiB)
 void zvc_compress_scratch(uint64_t n, int w, uint64_t F, uint64_t* tiles, uint64_t* aux) {
   const uint64_t TILE = 16384 / w, K = cdiv(n, F), tpf = cdiv(F, TILE);
-  *tiles = K ? (K - 1) * tpf + cdiv(frame_len(n, F, K - 1), TILE) : 0;
+  *tiles = (K ? (K - 1) * tpf + cdiv(frame_len(n, F, K - 1), TILE) : 0) * kStatusStride;
   // sc.zacc: frame + group accumulators, fdone, CTA counter, kAccStride words apart
   *aux = (2 * K + K * ((tpf + 31) / 32) + 2) * kAccStride;
 }
