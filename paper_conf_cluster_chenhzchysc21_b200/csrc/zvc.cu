@@ -109,6 +109,13 @@ constexpr uint64_t kAccStride = CSWAP_ZVC_ACC_STRIDE;
 #define CSWAP_ZVC_STATUS_STRIDE 2
 #endif
 constexpr uint64_t kStatusStride = CSWAP_ZVC_STATUS_STRIDE;
+// 1: a per-frame accumulator (one atomic per tile) gives the next frame its start; 0: the next
+// frame's first resolver sums the frame's 32-tile group accumulators instead (one hot word and
+// one atomic per tile fewer; A/B x2, profiles/zvc_frameacc_ab_r02.jsonl: f16 1 GiB -1..1.5 %,
+// f32 0..-0.7 %)
+#ifndef CSWAP_ZVC_FRAMEACC
+#define CSWAP_ZVC_FRAMEACC 0
+#endif
 #ifndef CSWAP_ZVC_POW2
 #define CSWAP_ZVC_POW2 1
 #endif
@@ -383,7 +390,29 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
       // offset = frame start + bitmap + W * (totals of earlier 32-tile groups of the frame +
       // counts of earlier tiles of the group).  Everything comes from COUNTS (published as soon
       // as a tile lands), never from other tiles' resolutions, so no chain forms across tiles.
-      if (j == 0 && lane == 0) {
+      if (!CSWAP_ZVC_FRAMEACC && j == 0 && k > 0) {
+        // previous frame's start + its bitmap + its packed values, the values summed from the
+        // previous frame's group accumulators (lane l: groups l, l + 32, ...), each complete
+        const uint64_t Fp = frame_len(n, F, k - 1);
+        const uint32_t tiles_prev = uint32_t(cdiv(Fp, G::TILE)), gp = (tiles_prev + 31) / 32;
+        uint64_t nz = 0;
+        for (uint32_t gi = lane; gi < gp; gi += 32) {
+          const uint64_t* p = sc.zacc + (K + uint64_t(k - 1) * gpf + gi) * kAccStride;
+          const uint64_t want = gi + 1 < gp ? 32 : tiles_prev - 32 * gi;
+          uint64_t v;
+          uint32_t backoff = kMinBackoff;
+          while (((v = ld_relaxed(p)) >> 40) != want) resolver_pause(backoff);
+          nz += v & ((1ull << 40) - 1);
+        }
+        nz = warp_sum_u64(nz);
+        if (lane == 0) {
+          uint64_t a;
+          uint32_t backoff = kMinBackoff;
+          while (status_flag(a = ld_relaxed(sc.aux + k - 1), epoch) != kFlagP) resolver_pause(backoff);
+          fstart = status_value(a) + a16(4 * cdiv(Fp, 32)) + a16(G::W * nz);
+          st_relaxed(sc.aux + k, make_status(fstart, epoch, kFlagP));
+        }
+      } else if (j == 0 && lane == 0) {
         if (k == 0) {
           fstart = data_start(K);
         } else {  // previous frame's start + its bitmap + its packed values (from its accumulator)
@@ -566,7 +595,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
 #pragma unroll
       for (int w = 0; w < CW; w++) tot += s_wtot[s][w];
       st_relaxed(sc.status + uint64_t(t) * kStatusStride, make_status(tot, epoch, kFlagA));  // self-contained: no release needed
-      atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + k * kAccStride), (1ull << 40) + tot);
+      if (CSWAP_ZVC_FRAMEACC) atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + k * kAccStride), (1ull << 40) + tot);
       atomicAdd(reinterpret_cast<unsigned long long*>(sc.zacc + (K + uint64_t(k) * gpf + j / 32) * kAccStride),
                 (1ull << 40) + tot);
       s_nnz[s] = tot;
