@@ -590,7 +590,7 @@ __global__ void __launch_bounds__(compress_threads<S, CW>(), CompressSmem<T, S, 
                                                         : count_slab(std::false_type{}, stage, gsrc, te, be, bm_out);
     if (lane == 0) s_wtot[s][warp] = c;
     consumer_sync();
-    if (tid == 0) {  // publish the tile count (A) and feed the frame / group accumulators
+    if (tid == 0) {  // publish the tile count (A) and feed the group accumulator
       uint32_t tot = 0;
 #pragma unroll
       for (int w = 0; w < CW; w++) tot += s_wtot[s][w];
