@@ -52,6 +52,13 @@ struct Scratch {
   uint64_t* kclock;
 };
 
+// programmatic dependent launch: wait until the preceding kernel in the stream has completed and
+// its memory is visible (a no-op when the kernel was launched without the PDL attribute)
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+// let the next kernel of the stream (launched with the PDL attribute) start now: its CTAs become
+// resident and block in pdl_wait() until this grid has completed
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ uint64_t globaltimer_ns() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));

@@ -116,6 +116,10 @@ constexpr uint64_t kStatusStride = CSWAP_ZVC_STATUS_STRIDE;
 #ifndef CSWAP_ZVC_FRAMEACC
 #define CSWAP_ZVC_FRAMEACC 0
 #endif
+// decode chain: each kernel triggers its dependent's launch as it starts (PDL)
+#ifndef CSWAP_PDL_TRIGGER
+#define CSWAP_PDL_TRIGGER 1
+#endif
 #ifndef CSWAP_ZVC_POW2
 #define CSWAP_ZVC_POW2 1
 #endif
@@ -726,6 +730,8 @@ __global__ void __launch_bounds__(kThreads) zvc_count_kernel(const uint8_t* __re
   using G = ZvcGeom<T>;
   const int lane = threadIdx.x & 31;
   const uint32_t tl = blockIdx.x * kWarps + (threadIdx.x >> 5);
+  if (CSWAP_PDL_TRIGGER) pdl_trigger();
+  pdl_wait();  // prep's frame starts / sizes and error word
   if (tl >= num_tiles || *reinterpret_cast<volatile const uint32_t*>(err)) return;
   const uint32_t t = tl + k0 * tpf;
   const uint32_t k = t / tpf, j = t % tpf;
@@ -770,6 +776,8 @@ __global__ void __launch_bounds__(1024) zvc_scan_kernel(uint64_t n, uint64_t F, 
                                                         uint32_t* err) {
   using G = ZvcGeom<T>;
   __shared__ uint64_t s_w[33];
+  if (CSWAP_PDL_TRIGGER) pdl_trigger();
+  pdl_wait();  // the count kernel's tile counts
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const uint32_t k = k0 + blockIdx.x;
   const uint64_t Fk = frame_len(n, F, k);
@@ -816,12 +824,13 @@ __global__ void __launch_bounds__(kThreads) zvc_expand_kernel(const uint8_t* __r
   __shared__ uint32_t s_woff[kWarps];
   extern __shared__ __align__(16) uint8_t s_val[];  // kTileBytes + 32
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const uint32_t t = blockIdx.x + k0 * tpf;
   const uint32_t k = t / tpf, j = t % tpf;
   const uint64_t Fk = frame_len(n, F, k);
   const uint32_t tile_elems = uint32_t(umin64(G::TILE, Fk - uint64_t(j) * G::TILE));
   const uint32_t nw = (tile_elems + 31) / 32;
+  pdl_wait();  // the scan kernel's value offsets
+  if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const uint64_t fstart = sc.aux[k], fend = fstart + sc.aux2[k];
   const uint64_t vbeg = sc.tbuf[t];
   const uint64_t vend = (j + 1 < uint32_t(cdiv(Fk, G::TILE))) ? sc.tbuf[t + 1] : 0;  // next tile's start
@@ -996,6 +1005,36 @@ static int prof_enabled() {
   return p;
 }
 
+// CSWAP_PDL=0: plain launches for the decode chain (A/B)
+static bool pdl_enabled() {
+  static int p = -1;
+  if (p < 0) {
+    const char* e = getenv("CSWAP_PDL");
+    p = (e && e[0] == '0') ? 0 : 1;
+  }
+  return p == 1;
+}
+template <typename... KArgs, typename... Args>
+static cudaError_t pdl_launch(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+#define CUDA_TRY_LAUNCH(x)                    \
+  do {                                        \
+    const cudaError_t e_ = (x);               \
+    if (e_ != cudaSuccess) return e_;         \
+  } while (0)
+
 // CSWAP_ZVC_COOP=0 launches the persistent compress non-cooperatively (A/B measurements only:
 // without it the kernel can stall behind concurrent kernels)
 static bool coop_enabled() {
@@ -1138,15 +1177,19 @@ static cudaError_t launch_zvc_decompress_t(const uint8_t* in, void* out, uint64_
   const uint32_t tiles = zvc_tiles(n, sizeof(T), F, k0, k1, &tpf);
   if (!tiles) return cudaSuccess;
   timing_kernel_start(st);
-  zvc_count_kernel<T><<<(tiles + kWarps - 1) / kWarps, kThreads, 0, st>>>(in, n, F, tpf, k0, tiles, sc, err);
-  zvc_scan_kernel<T><<<k1 - k0, 1024, 0, st>>>(n, F, tpf, k0, sc, err);
   const int smem = kTileBytes + 32;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(zvc_expand_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
-  zvc_expand_kernel<T><<<tiles, kThreads, smem, st>>>(in, static_cast<T*>(out), n, F, tpf, k0, sc, err);
+  // programmatic dependent launch: each kernel of the chain may be launched while its
+  // predecessor's last CTAs drain, and waits (griddepcontrol.wait) before reading its outputs
+  CUDA_TRY_LAUNCH(pdl_launch(zvc_count_kernel<T>, dim3((tiles + kWarps - 1) / kWarps), dim3(kThreads), 0, st, in, n,
+                             F, tpf, k0, tiles, sc, err));
+  CUDA_TRY_LAUNCH(pdl_launch(zvc_scan_kernel<T>, dim3(k1 - k0), dim3(1024), 0, st, n, F, tpf, k0, sc, err));
+  CUDA_TRY_LAUNCH(pdl_launch(zvc_expand_kernel<T>, dim3(tiles), dim3(kThreads), smem, st, in, static_cast<T*>(out), n,
+                             F, tpf, k0, sc, err));
   return cudaGetLastError();
 }
 
