@@ -3,6 +3,7 @@
 // Container v1 geometry, the epoch-tagged per-tile status words polled by the
 // persistent ZVC compress, TMA bulk-copy / mbarrier wrappers and small PTX memory-order helpers.
 #pragma once
+#include <cstdlib>
 #include <cstdint>
 #include <type_traits>
 #include <cuda_runtime.h>
@@ -254,5 +255,37 @@ __device__ __forceinline__ void write_header(uint8_t* out, int codec, int dtype,
   o64[6] = 0;
   o64[7] = 0;
 }
+
+// Programmatic dependent launch (PDL) for the kernels of a launch group: CSWAP_PDL=0 launches plainly (A/B).
+// Every kernel launched this way calls pdl_wait() before reading its predecessor's output.
+inline bool pdl_enabled() {
+  static int p = -1;
+  if (p < 0) {
+    const char* e = getenv("CSWAP_PDL");
+    p = (e && e[0] == '0') ? 0 : 1;
+  }
+  return p == 1;
+}
+template <typename... KArgs, typename... Args>
+inline cudaError_t pdl_launch(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+#define CUDA_TRY_LAUNCH(x)                    \
+  do {                                        \
+    const cudaError_t e_ = (x);               \
+    if (e_ != cudaSuccess) return e_;         \
+  } while (0)
+
 
 }  // namespace cswap

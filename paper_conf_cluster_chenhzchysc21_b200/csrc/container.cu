@@ -51,6 +51,8 @@ cudaError_t launch_none_compress(const void* in, uint64_t n, int w, uint64_t F, 
 __global__ void __launch_bounds__(1024) finalize_kernel(uint8_t* out, int codec, int dtype, uint64_t n, uint64_t F,
                                                         uint32_t param, const uint64_t* fbytes, uint64_t* fstart,
                                                         uint64_t* out_size) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   __shared__ uint64_t s_w[33];
   const uint32_t K = uint32_t(cdiv(n, F));
   const uint64_t base = data_start(K);
@@ -94,7 +96,7 @@ __global__ void __launch_bounds__(1024) finalize_kernel(uint8_t* out, int codec,
 
 cudaError_t launch_finalize(uint8_t* out, int codec, int dtype, uint64_t n, uint64_t F, uint32_t param,
                             const Scratch& sc, uint64_t* out_size, cudaStream_t st) {
-  finalize_kernel<<<1, 1024, 0, st>>>(out, codec, dtype, n, F, param, sc.aux2, sc.aux, out_size);
+  CUDA_TRY_LAUNCH(pdl_launch(finalize_kernel, dim3(1), dim3(1024), 0, st, out, codec, dtype, n, F, param, sc.aux2, sc.aux, out_size));
   return cudaGetLastError();
 }
 
@@ -114,12 +116,14 @@ cudaError_t launch_zero_words(void* p, uint64_t words, cudaStream_t st) {
 
 // ---- error word merge (device scratch word -> caller's word, first error wins) ---------------
 __global__ void err_merge_kernel(const uint32_t* src, uint32_t* dst) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   const uint32_t v = *src;
   if (v) atomicCAS(dst, 0u, v);
 }
 
 cudaError_t launch_err_merge(const uint32_t* src, uint32_t* dst, cudaStream_t st) {
-  err_merge_kernel<<<1, 1, 0, st>>>(src, dst);
+  CUDA_TRY_LAUNCH(pdl_launch(err_merge_kernel, dim3(1), dim3(1), 0, st, src, dst));
   return cudaGetLastError();
 }
 
@@ -153,6 +157,8 @@ __device__ __forceinline__ uint64_t block_excl_scan_u64(uint64_t v, uint64_t* s_
 __global__ void __launch_bounds__(1024) prep_kernel(const uint8_t* in, uint64_t in_size, int codec, int dtype,
                                                     uint64_t n, uint64_t F, uint32_t param, uint64_t* fstart,
                                                     uint64_t* fbytes, uint32_t* err, int reset_err) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   __shared__ int s_ok;
   __shared__ uint64_t s_total;
   __shared__ uint64_t s_warp[33];
@@ -208,7 +214,7 @@ __global__ void __launch_bounds__(1024) prep_kernel(const uint8_t* in, uint64_t 
 cudaError_t launch_prep(const uint8_t* in, uint64_t in_size, int codec, int dtype, uint64_t n, uint64_t F,
                         uint32_t param, const Scratch& sc, uint32_t* err, bool reset_err, cudaStream_t st) {
   timing_kernel_start(st);
-  prep_kernel<<<1, 1024, 0, st>>>(in, in_size, codec, dtype, n, F, param, sc.aux, sc.aux2, err, reset_err ? 1 : 0);
+  CUDA_TRY_LAUNCH(pdl_launch(prep_kernel, dim3(1), dim3(1024), 0, st, in, in_size, codec, dtype, n, F, param, sc.aux, sc.aux2, err, reset_err ? 1 : 0));
   return cudaGetLastError();
 }
 
@@ -324,6 +330,8 @@ namespace cswap {
 // last kernel, so every frame is complete; writes kProgReady | end offset of each frame from the
 // container's frame table (one CTA: per-thread chunk sums, block scan, per-thread writes).
 __global__ void __launch_bounds__(1024) publish_frames_kernel(const uint8_t* out, uint32_t K, uint64_t* prog) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   __shared__ uint64_t s_w[33];
   const uint64_t* fb = reinterpret_cast<const uint64_t*>(out + 64);
   const uint32_t per = (K + blockDim.x - 1) / blockDim.x, k0 = threadIdx.x * per, k1 = umin32(K, k0 + per);
@@ -356,7 +364,7 @@ __global__ void __launch_bounds__(1024) publish_frames_kernel(const uint8_t* out
 
 cudaError_t launch_publish_frames(const uint8_t* out, uint32_t K, uint64_t* prog, cudaStream_t st) {
   if (!K) return cudaSuccess;
-  publish_frames_kernel<<<1, 1024, 0, st>>>(out, K, prog);
+  CUDA_TRY_LAUNCH(pdl_launch(publish_frames_kernel, dim3(1), dim3(1024), 0, st, out, K, prog));
   return cudaGetLastError();
 }
 }  // namespace cswap

@@ -22,6 +22,8 @@ namespace cswap {
 template <typename T>
 __global__ void __launch_bounds__(kThreads) csr_count_kernel(const T* __restrict__ in, uint64_t n, uint64_t F,
                                                              uint32_t tpf, Scratch sc) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   using G = TileGeom<T>;
   __shared__ uint32_t s_tmp[33];
   const uint32_t t = blockIdx.x;
@@ -61,6 +63,8 @@ __global__ void __launch_bounds__(kThreads) csr_count_kernel(const T* __restrict
 template <typename T>
 __global__ void __launch_bounds__(1024) csr_scan_kernel(uint64_t n, uint64_t F, uint32_t tpf, uint32_t C,
                                                         Scratch sc) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   using G = TileGeom<T>;
   __shared__ uint64_t s_tmp[33];
   const uint32_t k = blockIdx.x;
@@ -87,6 +91,8 @@ template <typename T>
 __global__ void __launch_bounds__(kThreads) csr_emit_kernel(const T* __restrict__ in, uint64_t n, uint64_t F,
                                                             uint32_t tpf, uint32_t C, uint8_t* __restrict__ out,
                                                             Scratch sc) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   using G = TileGeom<T>;
   __shared__ uint32_t s_wcnt[kWarps + 1];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -198,11 +204,11 @@ static cudaError_t csr_compress_t(const void* in, uint64_t n, uint64_t F, uint32
   const uint32_t tiles = rle_tiles(n, sizeof(T), F);
   const T* x = static_cast<const T*>(in);
   timing_kernel_start(st);
-  csr_count_kernel<T><<<tiles, kThreads, 0, st>>>(x, n, F, tpf, sc);
-  csr_scan_kernel<T><<<K, 1024, 0, st>>>(n, F, tpf, C, sc);
+  CUDA_TRY_LAUNCH(pdl_launch(csr_count_kernel<T>, dim3(tiles), dim3(kThreads), 0, st, x, n, F, tpf, sc));
+  CUDA_TRY_LAUNCH(pdl_launch(csr_scan_kernel<T>, dim3(K), dim3(1024), 0, st, n, F, tpf, C, sc));
   cudaError_t e = launch_finalize(out, kCSR, dtype, n, F, C, sc, out_size, st);
   if (e != cudaSuccess) return e;
-  csr_emit_kernel<T><<<tiles, kThreads, 0, st>>>(x, n, F, tpf, C, out, sc);
+  CUDA_TRY_LAUNCH(pdl_launch(csr_emit_kernel<T>, dim3(tiles), dim3(kThreads), 0, st, x, n, F, tpf, C, out, sc));
   return cudaGetLastError();
 }
 
@@ -222,6 +228,8 @@ template <typename T>
 __global__ void __launch_bounds__(kThreads) csr_expand_kernel(const uint8_t* __restrict__ in, T* __restrict__ outp,
                                                               uint64_t n, uint64_t F, uint32_t tpf, uint32_t C,
                                                               uint32_t k0, Scratch sc, uint32_t* err) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   using G = TileGeom<T>;
   __shared__ __align__(16) T s_x[G::TILE];
   __shared__ int s_bad;
@@ -332,9 +340,9 @@ cudaError_t launch_csr_decompress(const uint8_t* in, void* out, uint64_t n, int 
   const uint32_t tiles = (k1 - 1 - k0) * tpf + uint32_t(cdiv(frame_len(n, F, k1 - 1), TILE));
   timing_kernel_start(st);
   if (w == 4)
-    csr_expand_kernel<uint32_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint32_t*>(out), n, F, tpf, C, k0, sc, err);
+    CUDA_TRY_LAUNCH(pdl_launch(csr_expand_kernel<uint32_t>, dim3(tiles), dim3(kThreads), 0, st, in, static_cast<uint32_t*>(out), n, F, tpf, C, k0, sc, err));
   else
-    csr_expand_kernel<uint16_t><<<tiles, kThreads, 0, st>>>(in, static_cast<uint16_t*>(out), n, F, tpf, C, k0, sc, err);
+    CUDA_TRY_LAUNCH(pdl_launch(csr_expand_kernel<uint16_t>, dim3(tiles), dim3(kThreads), 0, st, in, static_cast<uint16_t*>(out), n, F, tpf, C, k0, sc, err));
   return cudaGetLastError();
 }
 

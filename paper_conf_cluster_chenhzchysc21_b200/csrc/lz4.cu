@@ -84,6 +84,8 @@ __device__ __forceinline__ uint32_t le32_g(const uint8_t* s, uint32_t p) {  // s
 __global__ void __launch_bounds__(32 * kLz4Warps) lz4_compress_kernel(const uint8_t* __restrict__ in, uint64_t n,
                                                                       int w, uint64_t F, uint32_t B, uint32_t bpf,
                                                                       uint32_t nblk, uint8_t* slots, uint64_t* csize) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   __shared__ uint16_t s_tabs[kLz4Warps][4096];
   const int lane = threadIdx.x & 31;
   const uint32_t blk = blockIdx.x * kLz4Warps + (threadIdx.x >> 5);
@@ -148,6 +150,8 @@ __global__ void __launch_bounds__(32 * kLz4Warps) lz4_compress_kernel(const uint
 // one CTA per frame: block offsets inside the frame's block section (tbuf), frame_bytes (aux2)
 __global__ void __launch_bounds__(1024) lz4_scan_kernel(uint64_t n, int w, uint64_t F, uint32_t B, uint32_t bpf,
                                                         Scratch sc) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   __shared__ uint64_t s_tmp[33];
   const uint32_t k = blockIdx.x;
   const uint32_t nb = uint32_t(cdiv(frame_len(n, F, k) * uint64_t(w), B));
@@ -168,6 +172,8 @@ __global__ void __launch_bounds__(1024) lz4_scan_kernel(uint64_t n, int w, uint6
 // one CTA per block: copy the slot to its place, write csize[b], pads
 __global__ void __launch_bounds__(256) lz4_pack_kernel(uint64_t n, int w, uint64_t F, uint32_t B, uint32_t bpf,
                                                        const uint8_t* slots, uint8_t* out, Scratch sc) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   const uint32_t blk = blockIdx.x;
   const uint32_t k = blk / bpf, b = blk % bpf;
   const uint32_t nb = uint32_t(cdiv(frame_len(n, F, k) * uint64_t(w), B));
@@ -204,12 +210,12 @@ cudaError_t launch_lz4_compress(const void* in, uint64_t n, int w, uint64_t F, u
   uint32_t bpf;
   const uint32_t nblk = lz4_blocks(n, w, F, B, &bpf);
   timing_kernel_start(st);
-  lz4_compress_kernel<<<(nblk + kLz4Warps - 1) / kLz4Warps, 32 * kLz4Warps, 0, st>>>(
-      static_cast<const uint8_t*>(in), n, w, F, B, bpf, nblk, slots, sc.tbuf);
-  lz4_scan_kernel<<<K, 1024, 0, st>>>(n, w, F, B, bpf, sc);
+  CUDA_TRY_LAUNCH(pdl_launch(lz4_compress_kernel, dim3((nblk + kLz4Warps - 1) / kLz4Warps), dim3(32 * kLz4Warps), 0, st, 
+      static_cast<const uint8_t*>(in), n, w, F, B, bpf, nblk, slots, sc.tbuf));
+  CUDA_TRY_LAUNCH(pdl_launch(lz4_scan_kernel, dim3(K), dim3(1024), 0, st, n, w, F, B, bpf, sc));
   cudaError_t e = launch_finalize(out, kLZ4, dtype, n, F, B, sc, out_size, st);
   if (e != cudaSuccess) return e;
-  lz4_pack_kernel<<<nblk, 256, 0, st>>>(n, w, F, B, bpf, slots, out, sc);
+  CUDA_TRY_LAUNCH(pdl_launch(lz4_pack_kernel, dim3(nblk), dim3(256), 0, st, n, w, F, B, bpf, slots, out, sc));
   return cudaGetLastError();
 }
 
@@ -220,6 +226,8 @@ cudaError_t launch_lz4_compress(const void* in, uint64_t n, int w, uint64_t F, u
 __global__ void __launch_bounds__(1024) lz4_dscan_kernel(const uint8_t* __restrict__ in, uint64_t n, int w,
                                                          uint64_t F, uint32_t B, uint32_t bpf, uint32_t k0, Scratch sc,
                                                          uint32_t* err) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   __shared__ uint64_t s_tmp[33];
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const uint32_t k = k0 + blockIdx.x;
@@ -260,6 +268,8 @@ __global__ void __launch_bounds__(32 * kLz4Warps) lz4_decode_kernel(const uint8_
                                                                     uint64_t n, int w, uint64_t F, uint32_t B,
                                                                     uint32_t bpf, uint32_t k0, uint32_t nslots,
                                                                     Scratch sc, uint32_t* err) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   // the warp's last kLz4Ring output bytes (ring indexed by output position): match sources within
   // that distance are read from shared memory, not back from L2 (an L2 round trip per match
   // bounded the decode at ~55 GB/s for ReLU data, whose matches are mostly a few bytes back)
@@ -363,10 +373,10 @@ cudaError_t launch_lz4_decompress(const uint8_t* in, void* out, uint64_t n, int 
   if (k1 <= k0) return cudaSuccess;
   const uint32_t bpf = uint32_t(cdiv(F * w, B));
   timing_kernel_start(st);
-  lz4_dscan_kernel<<<k1 - k0, 1024, 0, st>>>(in, n, w, F, B, bpf, k0, sc, err);
+  CUDA_TRY_LAUNCH(pdl_launch(lz4_dscan_kernel, dim3(k1 - k0), dim3(1024), 0, st, in, n, w, F, B, bpf, k0, sc, err));
   const uint32_t nslots = (k1 - k0) * bpf;
-  lz4_decode_kernel<<<(nslots + kLz4Warps - 1) / kLz4Warps, 32 * kLz4Warps, 0, st>>>(
-      in, static_cast<uint8_t*>(out), n, w, F, B, bpf, k0, nslots, sc, err);
+  CUDA_TRY_LAUNCH(pdl_launch(lz4_decode_kernel, dim3((nslots + kLz4Warps - 1) / kLz4Warps), dim3(32 * kLz4Warps), 0, st, 
+      in, static_cast<uint8_t*>(out), n, w, F, B, bpf, k0, nslots, sc, err));
   return cudaGetLastError();
 }
 

@@ -25,6 +25,8 @@ __device__ __forceinline__ bool run_start(const T* s_x, uint32_t e, const TilePo
 template <typename T>
 __global__ void __launch_bounds__(kThreads) rle_count_kernel(const T* __restrict__ in, uint64_t n, uint64_t F,
                                                              uint32_t tpf, Scratch sc) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   using G = TileGeom<T>;
   __shared__ __align__(16) T s_x[G::TILE];
   __shared__ uint64_t s_tmp[33];
@@ -53,6 +55,8 @@ __global__ void __launch_bounds__(kThreads) rle_count_kernel(const T* __restrict
 // r_k (aux3), frame_bytes (aux2)
 template <typename T>
 __global__ void __launch_bounds__(1024) rle_scan_kernel(uint64_t n, uint64_t F, uint32_t tpf, Scratch sc) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   using G = TileGeom<T>;
   __shared__ uint64_t s_tmp[33];
   const uint32_t k = blockIdx.x;
@@ -90,6 +94,8 @@ __global__ void __launch_bounds__(1024) rle_scan_kernel(uint64_t n, uint64_t F, 
 template <typename T>
 __global__ void __launch_bounds__(kThreads) rle_emit_kernel(const T* __restrict__ in, uint64_t n, uint64_t F,
                                                             uint32_t tpf, uint8_t* __restrict__ out, Scratch sc) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   using G = TileGeom<T>;
   __shared__ __align__(16) T s_x[G::TILE];
   __shared__ uint32_t s_wcnt[kWarps + 1];
@@ -175,8 +181,8 @@ static cudaError_t rle_compress_t(const void* in, uint64_t n, uint64_t F, uint8_
   const uint32_t tiles = rle_tiles(n, sizeof(T), F);
   const T* x = static_cast<const T*>(in);
   timing_kernel_start(st);
-  rle_count_kernel<T><<<tiles, kThreads, 0, st>>>(x, n, F, tpf, sc);
-  rle_scan_kernel<T><<<K, 1024, 0, st>>>(n, F, tpf, sc);
+  CUDA_TRY_LAUNCH(pdl_launch(rle_count_kernel<T>, dim3(tiles), dim3(kThreads), 0, st, x, n, F, tpf, sc));
+  CUDA_TRY_LAUNCH(pdl_launch(rle_scan_kernel<T>, dim3(K), dim3(1024), 0, st, n, F, tpf, sc));
   cudaError_t e = launch_finalize(out, kRLE, dtype, n, F, 0, sc, out_size, st);
   if (e != cudaSuccess) return e;
   const int smem = G::TILE * 2;
@@ -185,7 +191,7 @@ static cudaError_t rle_compress_t(const void* in, uint64_t n, uint64_t F, uint8_
     cudaFuncSetAttribute(rle_emit_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
-  rle_emit_kernel<T><<<tiles, kThreads, smem, st>>>(x, n, F, tpf, out, sc);
+  CUDA_TRY_LAUNCH(pdl_launch(rle_emit_kernel<T>, dim3(tiles), dim3(kThreads), smem, st, x, n, F, tpf, out, sc));
   return cudaGetLastError();
 }
 
@@ -220,6 +226,8 @@ __global__ void __launch_bounds__(kThreads) rle_dsum_kernel(const uint8_t* __res
                                                             int w, uint32_t k0, uint32_t k1, uint32_t cpf,
                                                             uint64_t* csum, uint32_t* npieces, Scratch sc,
                                                             uint32_t* err) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   if (blockIdx.x == 0 && threadIdx.x == 0) *npieces = 0;  // rle_runs_kernel appends long-run pieces
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const int lane = threadIdx.x & 31;
@@ -254,6 +262,8 @@ __global__ void __launch_bounds__(kThreads) rle_dsum_kernel(const uint8_t* __res
 __global__ void __launch_bounds__(1024) rle_dscan2_kernel(const uint8_t* __restrict__ in, uint64_t n, uint64_t F,
                                                           int w, uint32_t k0, uint32_t cpf, uint64_t* csum,
                                                           Scratch sc, uint32_t* err) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   __shared__ uint64_t s_tmp[33];
   __shared__ int s_ok;
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
@@ -300,6 +310,8 @@ __global__ void __launch_bounds__(kThreads) rle_runs_kernel(const uint8_t* __res
                                                             uint32_t cpf, const uint64_t* __restrict__ cstart,
                                                             RlePiece* pieces, uint32_t* npieces, uint64_t cap,
                                                             Scratch sc, uint32_t* err) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   __shared__ uint64_t s_wtot[kWarps];
   if (*reinterpret_cast<volatile const uint32_t*>(err)) return;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -375,6 +387,8 @@ __global__ void __launch_bounds__(kThreads) rle_runs_kernel(const uint8_t* __res
 template <typename T>
 __global__ void __launch_bounds__(kThreads) rle_fill_kernel(T* __restrict__ outp, const RlePiece* pieces,
                                                             const uint32_t* npieces) {
+  pdl_trigger();  // PDL: the next kernel of the group may launch now
+  pdl_wait();     // ... and this one reads its predecessor's output only after it completed
   const uint32_t total = *npieces;
   for (uint32_t p = blockIdx.x; p < total; p += gridDim.x) {
     const RlePiece pc = pieces[p];
@@ -416,21 +430,21 @@ cudaError_t launch_rle_decompress(const uint8_t* in, void* out, uint64_t n, int 
   RlePiece* pcs = reinterpret_cast<RlePiece*>(tmp + off_pc);
   timing_kernel_start(st);
   const uint64_t dgrid = std::min<uint64_t>(cdiv(slots, kWarps), 148 * 16);
-  rle_dsum_kernel<<<uint32_t(dgrid), kThreads, 0, st>>>(in, n, F, w, k0, k1, cpf, cs, cnt, sc, err);
-  rle_dscan2_kernel<<<k1 - k0, 1024, 0, st>>>(in, n, F, w, k0, cpf, cs, sc, err);
+  CUDA_TRY_LAUNCH(pdl_launch(rle_dsum_kernel, dim3(uint32_t(dgrid)), dim3(kThreads), 0, st, in, n, F, w, k0, k1, cpf, cs, cnt, sc, err));
+  CUDA_TRY_LAUNCH(pdl_launch(rle_dscan2_kernel, dim3(k1 - k0), dim3(1024), 0, st, in, n, F, w, k0, cpf, cs, sc, err));
 #ifndef CSWAP_RLE_RGRID
 #define CSWAP_RLE_RGRID (148 * 32)  // grid-stride CTAs of the run expansion (148 * 8: 6-14 % slower)
 #endif
   const uint32_t rgrid = uint32_t(CSWAP_RLE_RGRID ? std::min<uint64_t>(slots, CSWAP_RLE_RGRID) : slots);
   const uint32_t fgrid = 148 * 4;
   if (w == 4) {
-    rle_runs_kernel<uint32_t><<<rgrid, kThreads, 0, st>>>(in, static_cast<uint32_t*>(out), n, F, k0, k1, cpf, cs,
-                                                          pcs, cnt, cap, sc, err);
-    rle_fill_kernel<uint32_t><<<fgrid, kThreads, 0, st>>>(static_cast<uint32_t*>(out), pcs, cnt);
+    CUDA_TRY_LAUNCH(pdl_launch(rle_runs_kernel<uint32_t>, dim3(rgrid), dim3(kThreads), 0, st, in, static_cast<uint32_t*>(out), n, F, k0, k1, cpf, cs,
+                                                          pcs, cnt, cap, sc, err));
+    CUDA_TRY_LAUNCH(pdl_launch(rle_fill_kernel<uint32_t>, dim3(fgrid), dim3(kThreads), 0, st, static_cast<uint32_t*>(out), pcs, cnt));
   } else {
-    rle_runs_kernel<uint16_t><<<rgrid, kThreads, 0, st>>>(in, static_cast<uint16_t*>(out), n, F, k0, k1, cpf, cs,
-                                                          pcs, cnt, cap, sc, err);
-    rle_fill_kernel<uint16_t><<<fgrid, kThreads, 0, st>>>(static_cast<uint16_t*>(out), pcs, cnt);
+    CUDA_TRY_LAUNCH(pdl_launch(rle_runs_kernel<uint16_t>, dim3(rgrid), dim3(kThreads), 0, st, in, static_cast<uint16_t*>(out), n, F, k0, k1, cpf, cs,
+                                                          pcs, cnt, cap, sc, err));
+    CUDA_TRY_LAUNCH(pdl_launch(rle_fill_kernel<uint16_t>, dim3(fgrid), dim3(kThreads), 0, st, static_cast<uint16_t*>(out), pcs, cnt));
   }
   return cudaGetLastError();
 }

@@ -1005,36 +1005,6 @@ static int prof_enabled() {
   return p;
 }
 
-// CSWAP_PDL=0: plain launches for the decode chain (A/B)
-static bool pdl_enabled() {
-  static int p = -1;
-  if (p < 0) {
-    const char* e = getenv("CSWAP_PDL");
-    p = (e && e[0] == '0') ? 0 : 1;
-  }
-  return p == 1;
-}
-template <typename... KArgs, typename... Args>
-static cudaError_t pdl_launch(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
-                              Args... args) {
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = grid;
-  cfg.blockDim = block;
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = st;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
-  cfg.attrs = at;
-  cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
-}
-#define CUDA_TRY_LAUNCH(x)                    \
-  do {                                        \
-    const cudaError_t e_ = (x);               \
-    if (e_ != cudaSuccess) return e_;         \
-  } while (0)
-
 // CSWAP_ZVC_COOP=0 launches the persistent compress non-cooperatively (A/B measurements only:
 // without it the kernel can stall behind concurrent kernels)
 static bool coop_enabled() {
