@@ -87,7 +87,8 @@ for task in "$@"; do
     nvcc -gencode arch=compute_100a,code=sm_100a -O3 -shared -Xcompiler -fPIC tools/zc_probe.cu -o tools/zc_probe.so && timeout 300 python tools/zc_probe.py > gpurun_out/zc_probe.txt 2>&1
     nvcc -gencode arch=compute_100a,code=sm_100a -O2 -o /tmp/egp tools/event_gap_probe.cu && timeout 300 /tmp/egp > gpurun_out/event_gap_probe.txt 2>&1
     timeout 300 python tools/host_overhead_probe.py > gpurun_out/host_overhead.jsonl 2>&1
-    timeout 120 python tools/fresh_box_probe.py > gpurun_out/fresh_box_probe.jsonl 2>&1 ;;
+    timeout 120 python tools/fresh_box_probe.py > gpurun_out/fresh_box_probe.jsonl 2>&1
+    nvcc -gencode arch=compute_100a,code=sm_100a -O2 -o /tmp/dip tools/d2h_interference_probe.cu && timeout 300 /tmp/dip > gpurun_out/d2h_interference.jsonl 2>&1 ;;
   cpuplan)
     timeout 1800 python bench.py --cpu-plan gpurun_out/cpu_plan.json > gpurun_out/cpu_plan.log 2>&1 ;;
   *) echo "unknown task $task" ;;
