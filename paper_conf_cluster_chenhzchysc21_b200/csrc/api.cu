@@ -205,6 +205,10 @@ struct Ctx {
   // on a copy stream stalls that stream ~25-35 us while PCIe is busy, tools/event_probe.cu: the
   // other stream's copy keeps the link busy meanwhile)
   cudaStream_t s_d2h = nullptr, s_h2d = nullptr, s_h2d2 = nullptr;
+  // progress stream: copies a swap-out's device-side progress words to the host once its codec
+  // group is done (the codec kernels then store no host memory: a kernel that does completes only
+  // after its store drained behind the D2H queue, ~15-25 us of the caller's stream, §7.3)
+  cudaStream_t s_prog = nullptr;
   cudaMemPool_t pool = nullptr;  // private stream-ordered pool (staging, LZ4 slots, decode scratch)
   uint64_t* dev_sink = nullptr;  // device word for container sizes nobody reads
   // kernel-timing stamps (cswap_set_kernel_timing): a ring of 3-word slots in DEVICE memory.  A
@@ -811,6 +815,13 @@ struct OutJob {
 // placed in their pinned allocation so that `h->host` has a chosen residue mod 256 (the staging
 // buffer's, or the raw tensor's minus the data offset), and copies start at 256-aligned addresses.
 constexpr uintptr_t kDmaAlign = 256;
+// a swap-out whose frames are published at the end of its group: the group writes the progress
+// words to device memory and the progress stream copies them to the host (CSWAP_DEV_PROG=0: the
+// group stores them to host-mapped memory itself, A/B)
+#ifndef CSWAP_DEV_PROG
+#define CSWAP_DEV_PROG 1
+#endif
+constexpr bool kDevProg = CSWAP_DEV_PROG != 0;
 bool alloc_host(Ctx* c, cswap_handle* h, uint64_t bytes, uintptr_t residue) {
   h->host_base = c->pinned.alloc(bytes + kDmaAlign);
   if (!h->host_base) {
@@ -1067,6 +1078,7 @@ cswap_status cswap_init(int device) {
   CU(cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking));
   CU(cudaStreamCreateWithFlags(&c->s_h2d, cudaStreamNonBlocking));
   CU(cudaStreamCreateWithFlags(&c->s_h2d2, cudaStreamNonBlocking));
+  CU(cudaStreamCreateWithFlags(&c->s_prog, cudaStreamNonBlocking));
   for (auto& b : c->blocks) {
     CU(cudaEventCreateWithFlags(&b.ev, cudaEventDisableTiming));
     TRY(ensure_block(b, 1 << 16, 1 << 12));
@@ -1128,6 +1140,7 @@ cswap_status cswap_shutdown(void) {
   cudaStreamDestroy(c->s_d2h);
   cudaStreamDestroy(c->s_h2d);
   cudaStreamDestroy(c->s_h2d2);
+  cudaStreamDestroy(c->s_prog);
   c->pinned.destroy();
   c->small.destroy();
   delete c;
@@ -1520,9 +1533,14 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
   // staging placed so that its data start (staging + ds) is 256-aligned: the first copy of every
   // container starts aligned, later copies start at aligned addresses at or below their frame
   uint8_t* staging_base = nullptr;
-  if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging_base), cap + kDmaAlign, c->pool, st) != cudaSuccess)
+  const uint64_t prog_bytes = 8ull * std::max<uint32_t>(K, 1);
+  if (cudaMallocFromPoolAsync(reinterpret_cast<void**>(&staging_base), cap + 2 * kDmaAlign + prog_bytes, c->pool,
+                              st) != cudaSuccess)
     return bail(fail(CSWAP_ERR_NOMEM, "device staging of %llu B failed", (unsigned long long)cap));
   uint8_t* staging = staging_base + ((uintptr_t(0) - ds - addr(staging_base)) & (kDmaAlign - 1));
+  // device copy of the progress words, after the container (published by the group, copied to
+  // the host words on the progress stream once the group is done)
+  uint64_t* dprog = reinterpret_cast<uint64_t*>(staging + ((cap + kDmaAlign - 1) & ~uint64_t(kDmaAlign - 1)));
   // per-frame publication pays only when the D2H link would otherwise wait for this tensor's
   // compression (nothing queued ahead of it); CSWAP_FRAME_PUBLISH=0/1 forces it off/on.  Only
   // ZVC publishes from inside its kernel; then the host container is pinned at the worst case
@@ -1553,12 +1571,23 @@ cswap_status cswap_swap_out(const void* d_in, uint64_t n, cswap_dtype dtype, csw
     // the container size goes to the timer's pinned slot when timing (read at collection), else
     // to a device word nobody reads (the executor takes the size from the progress words)
     uint64_t* osz = tm.stamps ? tm.stamps + 2 : c->dev_sink;
-    s = do_compress(c, d_in, n, dtype, use, f, staging, osz, st, prog, frame_publish);
+    // frames published one by one from inside the kernel go straight to the host words; a group
+    // that publishes at its end writes device words, copied below
+    s = do_compress(c, d_in, n, dtype, use, f, staging, osz, st, (frame_publish || !kDevProg) ? prog : dprog,
+                    frame_publish);
     if (s == CSWAP_OK) tm.commit(use, 0, n * uint64_t(w), 0);
   }
   if (s == CSWAP_OK && (cudaEventCreateWithFlags(&done, cudaEventDisableTiming) != cudaSuccess ||
                         cudaEventRecord(done, st) != cudaSuccess))
     s = fail(CSWAP_ERR_CUDA, "event record failed");
+  if (s == CSWAP_OK && !frame_publish && kDevProg) {
+    // the progress words reach the host after the group: `done` is re-recorded behind the copy,
+    // so "group done" still implies "every word visible" for the executor
+    if (cudaStreamWaitEvent(c->s_prog, done, 0) != cudaSuccess ||
+        cudaMemcpyAsync(prog, dprog, prog_bytes, cudaMemcpyDeviceToHost, c->s_prog) != cudaSuccess ||
+        cudaEventRecord(done, c->s_prog) != cudaSuccess)
+      s = fail(CSWAP_ERR_CUDA, "progress copy failed");
+  }
   if (s != CSWAP_OK) {
     if (done) cudaEventDestroy(done);
     cudaFreeAsync(staging_base, st);
