@@ -41,9 +41,11 @@ struct Scratch {
   uint64_t* aux3;         // third per-frame u64 array (run / non-zero totals)
   uint64_t* zacc;         // persistent ZVC compress accumulators (zero between launches; cap_aux)
   uint64_t cap_tiles, cap_aux;
-  // swap-out progress (NULL outside cswap_swap_out): host-mapped pinned u64[K]; the compress
-  // group stores kProgReady | (end offset of frame k in the container) once every byte of frame
-  // k (and its frame-table entry) is in device memory, so the host can start that frame's D2H
+  // swap-out progress (NULL outside cswap_swap_out): u64[K], host-mapped pinned memory when
+  // frames are published one by one from inside the kernel, else device memory that the library
+  // copies to the host words after the group; the compress group stores kProgReady | (end offset
+  // of frame k in the container) once every byte of frame k (and its frame-table entry) is in
+  // device memory, so the host can start that frame's D2H
   uint64_t* prog;
   // ZVC compress only: 1 = publish each frame as soon as it is complete (the producer warps),
   // 2 = the last CTA publishes every frame once the kernel is done (no extra launch)
