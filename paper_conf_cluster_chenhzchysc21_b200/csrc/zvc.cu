@@ -90,7 +90,6 @@ __device__ __forceinline__ void resolver_pause(uint32_t& backoff) {
   __nanosleep(backoff);
   backoff = backoff < kMaxBackoff ? backoff * 2 : kMaxBackoff;
 }
-// rows per batch of count_slab's loads
 // accumulator words (per frame, per 32-tile group, per frame done-count, the CTA counter) are
 // CSWAP_ZVC_ACC_STRIDE u64 apart: 16 puts each on its own 128-byte line.  Packed, a frame's 16
 // group words shared one line that every consumer's atomics and every resolver's polls hit;
@@ -129,6 +128,7 @@ constexpr uint64_t kStatusStride = CSWAP_ZVC_STATUS_STRIDE;
 #ifndef CSWAP_ZVC_BM4
 #define CSWAP_ZVC_BM4 1
 #endif
+// rows per batch of count_slab's loads
 #ifndef CSWAP_ZVC_BATCH
 #define CSWAP_ZVC_BATCH 4
 #endif
