@@ -354,9 +354,10 @@ def _roofline(records, steps: int = 1) -> dict:
            "kernel": f"{names[codec]}_{'compress' if d == 0 else 'decompress'}", "launches": g["launches"],
            "algorithmic_bytes_per_launch": g["bytes"] / g["launches"], "avg_launch_ms": g["ms"] / g["launches"],
            "peak_source": src}
-    out["note"] = ("in-step CUDA events around each launch group include the event records' own cost while the "
-                   "concurrent D2H streams over PCIe (~25-35 us per record, tools/event_probe.cu, DESIGN.md §7.3); "
-                   "device_clock times the same launches with %globaltimer stamps, isolated without a copy running")
+    out["note"] = ("in-step CUDA events around each launch group include a timing event's own cost while the "
+                   "concurrent D2H streams over PCIe (~32 us of stream time per record, tools/event_gap_probe.cu, "
+                   "DESIGN.md §7.3); kernel_clock times the same compress launches by the kernel's own %globaltimer "
+                   "span, isolated the same tensors without a copy running")
     if g["dev_n"] == g["launches"] and g["dev_ms"] > 0:
         dev = g["bytes"] / (g["dev_ms"] * 1e-3) / 1e9
         out["device_clock"] = {
